@@ -1,0 +1,174 @@
+/*
+ * eim.h -- C ABI of the B200-native eIM hot path: IMM influence maximisation
+ * (Tang, Shi, Xiao, SIGMOD'15 = [22]) with GPU RRR-set sampling and greedy
+ * max-coverage seed selection, after Doney, Huang, Lee, "eIM", SC-W'25.
+ *
+ * Citations: "P:NNN" = line NNN of PAPER.md; "Rn" = reading n in DESIGN.md §3.
+ *
+ * Conventions (all entry points)
+ *   - Plain C types only.  Host input arrays are BORROWED for the duration of
+ *     the call (copied to the device); outputs are CALLER-ALLOCATED host
+ *     buffers.  The library owns every device allocation; eim_graph_free /
+ *     eim_destroy release them.
+ *   - Every call returns an eim_status; no exception or longjmp crosses the
+ *     ABI.  On failure eim_last_error(ctx) describes the cause; output
+ *     buffers are then unspecified unless stated otherwise.
+ *   - A context is single-threaded: do not call into one ctx concurrently.
+ *   - Results are pure functions of (graph, model, k, eps, ell, seed): they do
+ *     not depend on the device count, launch configuration or scheduling
+ *     (randomness is counter-based Philox keyed per sample and edge, R1).
+ *   - Graph: reverse CSR (CSC of the adjacency).  Row v lists the
+ *     in-neighbours u of v (edges u -> v) in ASCENDING order; position e in
+ *     in_neighbors is the edge id.  Self-loops and multi-edges are accepted
+ *     and count toward the in-degree d^-(v).
+ *   - Models use weighted-cascade weights p_uv = 1 / d^-(v)
+ *     (LT weights R3).
+ */
+#ifndef EIM_H
+#define EIM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  EIM_OK = 0,
+  EIM_E_INVAL = -1,     /* bad argument (see each call) */
+  EIM_E_NOMEM = -2,     /* device or host allocation failed */
+  EIM_E_CUDA = -3,      /* CUDA runtime error (message in eim_last_error) */
+  EIM_E_NCCL = -4,      /* NCCL error (multi-GPU contexts only) */
+  EIM_E_CAPACITY = -5,  /* caller buffer too small; required size is still reported */
+  EIM_E_STATE = -6      /* object used after free / wrong context */
+} eim_status;
+
+typedef enum { EIM_IC = 0, EIM_LT = 1 } eim_model;
+
+typedef struct eim_ctx eim_ctx;      /* one device, one stream, optional NCCL communicator */
+typedef struct eim_graph eim_graph;  /* device-resident reverse CSR + IC thresholds */
+
+/* Per-run statistics (nullable output of eim_imm_run). */
+typedef struct {
+  uint32_t rounds;              /* martingale rounds executed ([22] Alg. 2 loop) */
+  uint64_t theta_i[64];         /* |R| after round i */
+  uint64_t cov_i[64];           /* coverage of S_i on R after round i */
+  double lambda_p, lambda_s;    /* lambda' and lambda* ([22] Eq. 9 and 6) */
+  double lb;                    /* lower bound LB on OPT (1 if the loop never broke) */
+  uint64_t theta;               /* final |R| */
+  uint64_t cov;                 /* coverage of the final seed set */
+  uint64_t edges_examined;      /* IC: sum of d^-(u) over expanded u; LT: walk steps (local rank) */
+  uint64_t arena_elems;         /* members stored in R (all ranks) */
+  uint64_t tier2_samples;       /* samples redone in a global-memory tier (local rank) */
+  uint64_t kernel_launches;     /* eim kernels launched by this call (local rank) */
+  uint32_t sample_launches;     /* tier-1 sampler launches */
+  double ms_total;              /* wall time of the call (host clock) */
+  double ms_sample;             /* wall time in sampling (incl. retries, exchange) */
+  double ms_select;             /* wall time in greedy NodeSelection (incl. index build) */
+  double ms_comm;               /* wall time in NCCL exchanges */
+  double ms_sample_kernel;      /* device time of the tier-1 sampler kernels (CUDA events on the ctx stream) */
+} eim_stats;
+
+/* IMM parameters of [22] (host-only, no device needed). */
+typedef struct {
+  double ell_p;     /* l' = l (1 + ln 2 / ln n) */
+  double eps_p;     /* eps' = sqrt(2) eps */
+  double lnC;       /* ln binom(n, k), summed as sum_{i=1..k} ln(n-k+i) - ln i */
+  double lambda_p;  /* lambda' = (2 + 2/3 eps')(lnC + l' ln n + ln log2 n) n / eps'^2 */
+  double lambda_s;  /* lambda* = 2 n ((1-1/e) alpha + beta)^2 / eps^2 */
+  double log2n;     /* log2(n): the round loop runs while i < log2n */
+} eim_imm_params_t;
+
+#define EIM_NCCL_ID_BYTES 128
+
+/* ---------------------------------------------------------------- context
+ * eim_create: bind a context to CUDA `device`.  For world > 1 the caller
+ * runs one process per GPU, obtains an id from eim_nccl_get_id on rank 0,
+ * broadcasts its EIM_NCCL_ID_BYTES bytes (e.g. with torch.distributed) and
+ * passes it on every rank; the context then owns an NCCL communicator.
+ * `stream` is a cudaStream_t cast to uint64 (0 = the library creates its own
+ * non-blocking stream).  All device work of the context is issued on it.
+ * Errors: EIM_E_INVAL (device < 0, world < 1, rank not in [0, world),
+ * world > 1 without nccl_id), EIM_E_CUDA, EIM_E_NCCL, EIM_E_NOMEM.
+ */
+eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint64_t stream,
+                      eim_ctx** out);
+eim_status eim_nccl_get_id(void* out /* EIM_NCCL_ID_BYTES */);
+void eim_destroy(eim_ctx* ctx);
+/* Message for the last failed call on ctx (or for the last failed
+ * eim_create / host-only call when ctx is NULL).  Valid until the next call. */
+const char* eim_last_error(const eim_ctx* ctx);
+const char* eim_version(void);
+
+/* ---------------------------------------------------------------- graph
+ * eim_load_graph_csr: copy the reverse CSR to the device
+ * (replicated on every rank), validate it on the device and derive the IC
+ * thresholds T_v = floor((2^32-1) / d^-(v)) (R2: an edge into v is live iff
+ * its 32-bit draw <= T_v, i.e. P = 1/d^-(v)).
+ *   n: vertices, 2 <= n < 2^32 - 1.  m: edges, m < 2^40.
+ *   in_offsets[n+1]: in_offsets[0] = 0, non-decreasing, in_offsets[n] = m.
+ *   in_neighbors[m]: values < n.
+ * Pinned host buffers make the copies asynchronous and fast.
+ * Errors: EIM_E_INVAL for any violation above (nothing is kept), EIM_E_NOMEM,
+ * EIM_E_CUDA.
+ */
+eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                              const uint32_t* in_neighbors, eim_graph** out);
+eim_status eim_graph_free(eim_graph* g);
+
+/* ---------------------------------------------------------------- IMM
+ * eim_imm_run (Alg. 1, with [22] Alg. 2-3): theta estimation by the
+ * martingale loop, RRR sampling of sample ids 0..theta-1 (sets are reused
+ * across rounds and topped up, R14), and greedy NodeSelection.
+ *   k in [1, n]; eps in (0, 1); ell > 0 (IMM failure exponent, default 1).
+ *   seeds_out[k]: seed vertices in pick order.  theta_out: final |R|.
+ *   spread_out: n * cov / |R| (RIS estimate).  stats_out nullable.
+ * Multi-GPU contexts: every rank calls with identical arguments; each rank
+ * samples a contiguous share of every round's new ids, the shares are
+ * all-gathered over NCCL and the greedy runs replicated, so every rank
+ * returns the same result, identical to a single-GPU run.
+ * Errors: EIM_E_INVAL, EIM_E_STATE (graph from another ctx / freed),
+ * EIM_E_NOMEM, EIM_E_CUDA, EIM_E_NCCL.
+ */
+eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell,
+                       eim_model model, uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out,
+                       double* spread_out, eim_stats* stats_out);
+
+/* eim_sample_rrr (Alg. 2; LT P:134-140): RRR sets of sample ids
+ * [first_id, first_id + count), first_id + count <= 2^62, on this context's
+ * device (no communication).  Output in sample-id order, each set ascending
+ * (P:130): offsets_out[count+1] (offsets_out[0] = 0), members_out[<= cap].
+ * *members_total is always set to the number of members.  If members_cap is
+ * too small the call returns EIM_E_CAPACITY (offsets_out still valid,
+ * members_out unspecified).  Concatenating [a,b) and [b,c) gives [a,c).
+ */
+eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
+                          uint64_t first_id, uint64_t count, uint64_t* offsets_out,
+                          uint32_t* members_out, uint64_t members_cap, uint64_t* members_total);
+
+/* eim_select_seeds (Alg. 3): greedy max coverage of an arbitrary
+ * arena of num_sets sets over vertices [0, n): offsets[num_sets+1]
+ * (offsets[0] = 0, non-decreasing), members[offsets[num_sets]] (< n, no
+ * duplicates within a set; order within a set is free).  k in [1, n].
+ * seeds_out[k] in pick order; ties go to the lowest vertex id; when every
+ * set is covered the remaining picks are the lowest unselected ids (R10).
+ * gains_out[k] (nullable) = marginal coverage of each pick.
+ */
+eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const uint64_t* offsets,
+                            const uint32_t* members, uint32_t k, uint32_t* seeds_out,
+                            uint64_t* gains_out);
+
+/* ---------------------------------------------------------------- host-only
+ * These need no device and may be called with no context. */
+/* IMM parameters (formulas above; R17 fixes the evaluation order).
+ * Errors: EIM_E_INVAL if n < 2, k == 0, k > n, eps not in (0,1), ell <= 0. */
+eim_status eim_imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);
+/* Contiguous share of rank r among `world` ranks of the id range
+ * [first, first+count): [first + floor(r count / world), first + floor((r+1) count / world)). */
+eim_status eim_shard_range(uint64_t first, uint64_t count, int rank, int world, uint64_t* lo,
+                           uint64_t* hi);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EIM_H */

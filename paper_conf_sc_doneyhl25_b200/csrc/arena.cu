@@ -1,0 +1,148 @@
+// arena.cu -- the RRR arena R with per-set (start, length) (Fig. 2):
+// coverage histogram C, canonical export (sets in sample-id order,
+// each ascending) and appending sets received from other ranks.
+#include <cub/cub.cuh>
+
+#include "eim_internal.h"
+
+namespace eim {
+
+namespace {
+
+constexpr unsigned FULL = 0xFFFFFFFFu;
+
+// One warp per set: C[x] += 1 for every member x (sets have no duplicates).
+__global__ void hist_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,
+                            const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t hi,
+                            uint32_t* __restrict__ C) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t i = lo + warp; i < hi; i += nwarps) {
+    const uint64_t st = set_start[i];
+    const uint32_t L = set_len[i];
+    for (uint32_t t = lane; t < L; t += 32) atomicAdd(&C[arena[st + t]], 1u);
+  }
+}
+
+__global__ void len_to_u64_kernel(const uint32_t* __restrict__ len, uint64_t lo, uint64_t count,
+                                  uint64_t* __restrict__ out) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= count; i += stride)
+    out[i] = i < count ? (uint64_t)len[lo + i] : 0ull;
+}
+
+// One warp per set: copy arena[set_start[lo+i] ..] to out[offsets[i] ..].
+__global__ void gather_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,
+                              const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t count,
+                              const uint64_t* __restrict__ offsets, uint32_t* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t i = warp; i < count; i += nwarps) {
+    const uint64_t src = set_start[lo + i], dst = offsets[i];
+    const uint32_t L = set_len[lo + i];
+    for (uint32_t t = lane; t < L; t += 32) out[dst + t] = arena[src + t];
+  }
+}
+
+// Append canonical sets: members go to arena[base_elem + offsets[i] ..].
+__global__ void place_kernel(const uint64_t* __restrict__ offsets, uint64_t count, uint64_t base_set,
+                             uint64_t base_elem, uint64_t* __restrict__ set_start,
+                             uint32_t* __restrict__ set_len) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
+    set_start[base_set + i] = base_elem + offsets[i];
+    set_len[base_set + i] = (uint32_t)(offsets[i + 1] - offsets[i]);
+  }
+}
+
+}  // namespace
+
+void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi) {
+  if (hi <= lo) return;
+  hist_kernel<<<grid_for(ctx, (hi - lo) * 32, 256), 256, 0, ctx->stream>>>(
+      ctx->arena.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, hi,
+      ctx->C_total.as<uint32_t>());
+  EIM_CUDA(cudaGetLastError());
+  ctx->kernel_launches++;
+}
+
+// Compacts sets [lo, lo+count) (set indices) into stage_a (offsets, u64) and
+// stage_b (members).  Returns the member total.  sort: ascending within sets.
+static uint64_t compact_sets(eim_ctx* ctx, uint64_t lo, uint64_t count, bool sort, uint64_t** d_offsets,
+                             uint32_t** d_members) {
+  cudaStream_t st = ctx->stream;
+  ctx->stage_a.reserve((count + 1) * sizeof(uint64_t), false, st);
+  uint64_t* offs = ctx->stage_a.as<uint64_t>();
+  len_to_u64_kernel<<<grid_for(ctx, count + 1, 256), 256, 0, st>>>(ctx->set_len.as<uint32_t>(), lo, count, offs);
+  EIM_CUDA(cudaGetLastError());
+  size_t tmp = 0;
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, offs, offs, count + 1, st));
+  ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, offs, offs, count + 1, st));
+  uint64_t total = 0;
+  EIM_CUDA(cudaMemcpyAsync(ctx->h_pinned, offs + count, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+  total = *static_cast<uint64_t*>(ctx->h_pinned);
+  ctx->stage_b.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
+  uint32_t* out = ctx->stage_b.as<uint32_t>();
+  if (count > 0) {
+    gather_kernel<<<grid_for(ctx, count * 32, 256), 256, 0, st>>>(
+        ctx->arena.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, count, offs, out);
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches++;
+  }
+  ctx->kernel_launches += 1;
+  if (sort && total > 0) {
+    if (total > (uint64_t)INT32_MAX || count > (uint64_t)INT32_MAX)
+      fail(EIM_E_CAPACITY, "export larger than 2^31 members is not supported");
+    ctx->stage_c.reserve(total * sizeof(uint32_t), false, st);
+    uint32_t* sorted = ctx->stage_c.as<uint32_t>();
+    size_t tmp2 = 0;
+    EIM_CUDA(cub::DeviceSegmentedSort::SortKeys(nullptr, tmp2, out, sorted, (int)total, (int)count, offs,
+                                                 offs + 1, st));
+    ctx->scratch.reserve(std::max<size_t>(tmp2, 1 << 20), false, st);
+    EIM_CUDA(cub::DeviceSegmentedSort::SortKeys(ctx->scratch.p, tmp2, out, sorted, (int)total, (int)count,
+                                                 offs, offs + 1, st));
+    ctx->kernel_launches += 2;
+    out = sorted;
+  }
+  *d_offsets = offs;
+  *d_members = out;
+  return total;
+}
+
+uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members) {
+  return compact_sets(ctx, 0, count, true, d_offsets, d_members);
+}
+
+uint64_t compact_range(eim_ctx* ctx, uint64_t lo, uint64_t count, uint64_t** d_offsets, uint32_t** d_members) {
+  return compact_sets(ctx, lo, count, false, d_offsets, d_members);
+}
+
+void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_offsets,
+                 const uint32_t* d_members, uint64_t total) {
+  cudaStream_t st = ctx->stream;
+  if (count == 0) return;
+  ensure_sets(ctx, base + count);
+  uint64_t cur = arena_cursor(ctx);
+  const uint64_t cap = ctx->arena.bytes / sizeof(uint32_t);
+  if (cur + total > cap) ctx->arena.reserve(std::max<uint64_t>(cap * 2, cur + total) * sizeof(uint32_t), true, st);
+  if (total)
+    EIM_CUDA(cudaMemcpyAsync(ctx->arena.as<uint32_t>() + cur, d_members, total * sizeof(uint32_t),
+                             cudaMemcpyDeviceToDevice, st));
+  place_kernel<<<grid_for(ctx, count, 256), 256, 0, st>>>(d_offsets, count, base, cur,
+                                                           ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
+  EIM_CUDA(cudaGetLastError());
+  ctx->kernel_launches++;
+  // advance cursor and valid_end
+  unsigned long long* tail = reinterpret_cast<unsigned long long*>(ctx->ctl.as<SampleCtl>() + 1);
+  unsigned long long* h = static_cast<unsigned long long*>(ctx->h_pinned);
+  h[0] = cur + total;
+  h[1] = cur + total;
+  EIM_CUDA(cudaMemcpyAsync(tail, h, 2 * sizeof(unsigned long long), cudaMemcpyHostToDevice, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+}
+
+}  // namespace eim

@@ -1,0 +1,323 @@
+// capi.cpp -- the extern "C" boundary declared in include/eim.h: argument
+// validation, error capture (no exception crosses the ABI), object lifetime.
+#include <chrono>
+#include <cstring>
+#include <mutex>
+
+#include "eim_internal.h"
+
+namespace eim {
+
+void fail(eim_status code, const std::string& msg) { throw Error{code, msg}; }
+
+void cuda_check(cudaError_t e, const char* what, const char* file, int line) {
+  if (e == cudaSuccess) return;
+  const eim_status code = (e == cudaErrorMemoryAllocation) ? EIM_E_NOMEM : EIM_E_CUDA;
+  cudaGetLastError();  // clear sticky-free errors
+  fail(code, std::string(cudaGetErrorString(e)) + " in " + what + " (" + file + ":" + std::to_string(line) + ")");
+}
+
+void DevBuf::reserve(size_t need, bool keep, cudaStream_t st) {
+  if (need <= bytes) return;
+  size_t nb = std::max(need, bytes + bytes / 2);
+  nb = (nb + 255) & ~size_t(255);
+  void* q = nullptr;
+  cudaError_t e = cudaMalloc(&q, nb);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    nb = (need + 255) & ~size_t(255);
+    e = cudaMalloc(&q, nb);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      fail(EIM_E_NOMEM, "cudaMalloc of " + std::to_string(nb) + " bytes failed");
+    }
+  }
+  if (keep && p && bytes) {
+    EIM_CUDA(cudaMemcpyAsync(q, p, bytes, cudaMemcpyDeviceToDevice, st));
+    EIM_CUDA(cudaStreamSynchronize(st));
+  }
+  if (p) cudaFree(p);
+  p = q;
+  bytes = nb;
+}
+
+void DevBuf::release() {
+  if (p) cudaFree(p);
+  p = nullptr;
+  bytes = 0;
+}
+
+}  // namespace eim
+
+using namespace eim;
+
+namespace {
+
+std::mutex g_err_mu;
+std::string g_err;  // errors with no context
+
+void set_global_error(const std::string& m) {
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  g_err = m;
+}
+
+template <class F>
+eim_status guarded(eim_ctx* ctx, F&& f) {
+  try {
+    if (ctx) {
+      EIM_CUDA(cudaSetDevice(ctx->device));
+      ctx->last_error.clear();
+    }
+    f();
+    return EIM_OK;
+  } catch (const Error& e) {
+    if (ctx) ctx->last_error = e.msg;
+    else set_global_error(e.msg);
+    return e.code;
+  } catch (const std::bad_alloc&) {
+    if (ctx) ctx->last_error = "host allocation failed";
+    else set_global_error("host allocation failed");
+    return EIM_E_NOMEM;
+  } catch (...) {
+    if (ctx) ctx->last_error = "unknown error";
+    else set_global_error("unknown error");
+    return EIM_E_CUDA;
+  }
+}
+
+bool ctx_ok(const eim_ctx* ctx) { return ctx && ctx->magic == CTX_MAGIC; }
+
+void free_ctx_buffers(eim_ctx* c) {
+  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->retry_a, &c->retry_b,
+                    &c->tier_tab, &c->tier_queue, &c->tier_gen, &c->C_total, &c->C_work, &c->inv_off,
+                    &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
+                    &c->stage_b, &c->stage_c};
+  for (DevBuf* b : bufs) b->release();
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* eim_version(void) { return "eim-b200 0.1 (sm_100a)"; }
+
+const char* eim_last_error(const eim_ctx* ctx) {
+  if (ctx_ok(ctx)) return ctx->last_error.c_str();
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  return g_err.c_str();
+}
+
+eim_status eim_nccl_get_id(void* out) {
+  return guarded(nullptr, [&] {
+    if (!out) fail(EIM_E_INVAL, "out is NULL");
+    comm_get_id(out);
+  });
+}
+
+eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint64_t stream, eim_ctx** out) {
+  return guarded(nullptr, [&] {
+    if (!out) fail(EIM_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (device < 0) fail(EIM_E_INVAL, "device < 0");
+    if (world < 1 || rank < 0 || rank >= world) fail(EIM_E_INVAL, "rank/world out of range");
+    if (world > 1 && !nccl_id) fail(EIM_E_INVAL, "world > 1 needs an NCCL unique id");
+    int ndev = 0;
+    EIM_CUDA(cudaGetDeviceCount(&ndev));
+    if (device >= ndev) fail(EIM_E_INVAL, "device index out of range");
+    EIM_CUDA(cudaSetDevice(device));
+    eim_ctx* c = new eim_ctx();
+    c->magic = CTX_MAGIC;
+    c->device = device;
+    c->rank = rank;
+    c->world = world;
+    c->comm = nullptr;
+    c->kernel_launches = 0;
+    c->own_stream = stream == 0;
+    try {
+      if (c->own_stream) EIM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+      else c->stream = reinterpret_cast<cudaStream_t>(stream);
+      EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
+      EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
+      EIM_CUDA(cudaEventCreate(&c->ev0));
+      EIM_CUDA(cudaEventCreate(&c->ev1));
+      c->scratch.reserve(1 << 20, false, c->stream);
+      if (world > 1) c->comm = comm_create(rank, world, nccl_id);
+    } catch (...) {
+      free_ctx_buffers(c);
+      if (c->h_pinned) cudaFreeHost(c->h_pinned);
+      if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+      c->magic = 0;
+      delete c;
+      throw;
+    }
+    *out = c;
+  });
+}
+
+void eim_destroy(eim_ctx* ctx) {
+  if (!ctx_ok(ctx)) return;
+  cudaSetDevice(ctx->device);
+  cudaStreamSynchronize(ctx->stream);
+  comm_destroy(ctx->comm);
+  free_ctx_buffers(ctx);
+  cudaFreeHost(ctx->h_pinned);
+  cudaEventDestroy(ctx->ev0);
+  cudaEventDestroy(ctx->ev1);
+  if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
+  ctx->magic = 0;
+  delete ctx;
+}
+
+eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                              const uint32_t* in_neighbors, eim_graph** out) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  return guarded(ctx, [&] {
+    if (!out) fail(EIM_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (n < 2 || n >= 0xFFFFFFFFu) fail(EIM_E_INVAL, "n must be in [2, 2^32-1)");
+    if (m >= (1ull << 40)) fail(EIM_E_INVAL, "m must be < 2^40");
+    if (!in_offsets || (m > 0 && !in_neighbors)) fail(EIM_E_INVAL, "NULL graph array");
+    eim_graph* g = new eim_graph();
+    g->magic = GRAPH_MAGIC;
+    g->ctx = ctx;
+    cudaStream_t st = ctx->stream;
+    try {
+      EIM_CUDA(cudaMalloc(&g->d_off, ((uint64_t)n + 1) * sizeof(uint64_t)));
+      EIM_CUDA(cudaMalloc(&g->d_nbr, std::max<uint64_t>(m, 4) * sizeof(uint32_t)));
+      EIM_CUDA(cudaMalloc(&g->d_thr, (uint64_t)n * sizeof(uint32_t)));
+      EIM_CUDA(cudaMemcpyAsync(g->d_off, in_offsets, ((uint64_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+      if (m) EIM_CUDA(cudaMemcpyAsync(g->d_nbr, in_neighbors, m * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+      g->view.n = n;
+      g->view.m = m;
+      g->view.off = static_cast<const uint64_t*>(g->d_off);
+      g->view.nbr = static_cast<const uint32_t*>(g->d_nbr);
+      g->view.thr = static_cast<const uint32_t*>(g->d_thr);
+      graph_validate_and_thresholds(ctx, g);
+    } catch (...) {
+      cudaStreamSynchronize(st);
+      if (g->d_off) cudaFree(g->d_off);
+      if (g->d_nbr) cudaFree(g->d_nbr);
+      if (g->d_thr) cudaFree(g->d_thr);
+      g->magic = 0;
+      delete g;
+      throw;
+    }
+    *out = g;
+  });
+}
+
+eim_status eim_graph_free(eim_graph* g) {
+  if (!g || g->magic != GRAPH_MAGIC) return EIM_E_STATE;
+  eim_ctx* ctx = g->ctx;
+  if (ctx_ok(ctx)) {
+    cudaSetDevice(ctx->device);
+    cudaStreamSynchronize(ctx->stream);
+  }
+  cudaFree(g->d_off);
+  cudaFree(g->d_nbr);
+  cudaFree(g->d_thr);
+  g->magic = 0;
+  delete g;
+  return EIM_OK;
+}
+
+static void check_graph(eim_ctx* ctx, const eim_graph* g) {
+  if (!g || g->magic != GRAPH_MAGIC) fail(EIM_E_STATE, "graph is freed or invalid");
+  if (g->ctx != ctx) fail(EIM_E_STATE, "graph belongs to another context");
+}
+
+eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
+                       uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
+                       eim_stats* stats_out) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  return guarded(ctx, [&] {
+    check_graph(ctx, g);
+    if (!seeds_out) fail(EIM_E_INVAL, "seeds_out is NULL");
+    if (k == 0 || k > g->view.n) fail(EIM_E_INVAL, "k must be in [1, n]");
+    if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
+    if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
+    if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
+    eim_stats local;
+    imm_run(ctx, g, k, eps, ell, model, seed, seeds_out, theta_out, spread_out, stats_out ? stats_out : &local);
+  });
+}
+
+eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first_id,
+                          uint64_t count, uint64_t* offsets_out, uint32_t* members_out, uint64_t members_cap,
+                          uint64_t* members_total) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  eim_status cap_status = EIM_OK;
+  eim_status s = guarded(ctx, [&] {
+    check_graph(ctx, g);
+    if (!offsets_out || !members_total) fail(EIM_E_INVAL, "NULL output");
+    if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
+    if (first_id + count < first_id || first_id + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids must be < 2^62");
+    cudaStream_t st = ctx->stream;
+    arena_reset(ctx);
+    sample_range(ctx, g, model, seed, first_id, count, first_id, false);
+    uint64_t* d_off = nullptr;
+    uint32_t* d_mem = nullptr;
+    const uint64_t total = export_sets(ctx, count, &d_off, &d_mem);
+    *members_total = total;
+    EIM_CUDA(cudaMemcpyAsync(offsets_out, d_off, (count + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    if (total > members_cap) {
+      EIM_CUDA(cudaStreamSynchronize(st));
+      ctx->last_error = "members_cap too small";
+      cap_status = EIM_E_CAPACITY;
+      return;
+    }
+    if (total) {
+      if (!members_out) fail(EIM_E_INVAL, "members_out is NULL");
+      EIM_CUDA(cudaMemcpyAsync(members_out, d_mem, total * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    }
+    EIM_CUDA(cudaStreamSynchronize(st));
+  });
+  return s != EIM_OK ? s : cap_status;
+}
+
+eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const uint64_t* offsets,
+                            const uint32_t* members, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  return guarded(ctx, [&] {
+    if (n < 1 || n >= 0xFFFFFFFFu) fail(EIM_E_INVAL, "n must be in [1, 2^32-1)");
+    if (k == 0 || k > n) fail(EIM_E_INVAL, "k must be in [1, n]");
+    if (!offsets || !seeds_out) fail(EIM_E_INVAL, "NULL argument");
+    if (offsets[0] != 0) fail(EIM_E_INVAL, "offsets[0] != 0");
+    for (uint64_t i = 0; i < num_sets; ++i)
+      if (offsets[i + 1] < offsets[i]) fail(EIM_E_INVAL, "offsets not non-decreasing");
+    const uint64_t total = offsets[num_sets];
+    if (total && !members) fail(EIM_E_INVAL, "members is NULL");
+    for (uint64_t i = 0; i < total; ++i)
+      if (members[i] >= n) fail(EIM_E_INVAL, "member id >= n");
+    cudaStream_t st = ctx->stream;
+    arena_reset(ctx);
+    ctx->stage_a.reserve((num_sets + 1) * sizeof(uint64_t), false, st);
+    ctx->stage_b.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
+    EIM_CUDA(cudaMemcpyAsync(ctx->stage_a.p, offsets, (num_sets + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+    if (total) EIM_CUDA(cudaMemcpyAsync(ctx->stage_b.p, members, total * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+    ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, st);
+    EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), st));
+    append_sets(ctx, 0, num_sets, ctx->stage_a.as<uint64_t>(), ctx->stage_b.as<uint32_t>(), total);
+    hist_sets(ctx, 0, num_sets);
+    greedy(ctx, n, num_sets, k, seeds_out, gains_out);
+  });
+}
+
+eim_status eim_imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out) {
+  return guarded(nullptr, [&] {
+    if (!out) fail(EIM_E_INVAL, "out is NULL");
+    if (n < 2 || k == 0 || k > n || !(eps > 0.0 && eps < 1.0) || !(ell > 0.0))
+      fail(EIM_E_INVAL, "invalid IMM parameters");
+    imm_params(n, k, eps, ell, out);
+  });
+}
+
+eim_status eim_shard_range(uint64_t first, uint64_t count, int rank, int world, uint64_t* lo, uint64_t* hi) {
+  if (world < 1 || rank < 0 || rank >= world || !lo || !hi) return EIM_E_INVAL;
+  const unsigned __int128 c = count;
+  *lo = first + (uint64_t)(c * (unsigned)rank / (unsigned)world);
+  *hi = first + (uint64_t)(c * (unsigned)(rank + 1) / (unsigned)world);
+  return EIM_OK;
+}
+
+}  // extern "C"

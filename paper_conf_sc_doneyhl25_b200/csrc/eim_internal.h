@@ -1,0 +1,161 @@
+// eim_internal.h -- shared declarations of the CUDA path (never of the oracle).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "eim.h"
+
+namespace eim {
+
+// Thrown inside the library only; converted to eim_status at the ABI.
+struct Error {
+  eim_status code;
+  std::string msg;
+};
+
+[[noreturn]] void fail(eim_status code, const std::string& msg);
+void cuda_check(cudaError_t e, const char* what, const char* file, int line);
+#define EIM_CUDA(x) ::eim::cuda_check((x), #x, __FILE__, __LINE__)
+
+// Device buffer with geometric growth (contents optionally preserved).
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  void reserve(size_t need, bool keep, cudaStream_t st);
+  void release();
+  template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// Device-resident reverse CSR.
+struct GraphView {
+  uint32_t n;
+  uint64_t m;
+  const uint64_t* off;   // n+1
+  const uint32_t* nbr;   // m
+  const uint32_t* thr;   // n: IC threshold floor((2^32-1)/d), 0 if d == 0
+};
+
+// Where a sampler writes its sets.
+struct ArenaView {
+  uint32_t* elems;                 // members
+  unsigned long long* cursor;      // next free element
+  unsigned long long* valid_end;   // max end of a successful reservation
+  uint64_t cap;                    // capacity in elements
+  uint64_t* set_start;             // indexed by sample id - set_base
+  uint32_t* set_len;
+  uint64_t set_base;
+  uint32_t* C;                     // coverage histogram (nullable: no histogram)
+};
+
+// Per-launch control block (device memory).
+struct SampleCtl {
+  unsigned long long ticket;
+  unsigned long long retry_count;
+  unsigned long long edges;
+  unsigned long long arena_fail;
+};
+
+struct Comm;  // NCCL communicator wrapper (comm.cpp)
+
+}  // namespace eim
+
+struct eim_graph {
+  uint32_t magic;
+  eim_ctx* ctx;
+  eim::GraphView view;
+  void* d_off = nullptr;
+  void* d_nbr = nullptr;
+  void* d_thr = nullptr;
+};
+
+struct eim_ctx {
+  uint32_t magic;
+  int device, rank, world;
+  cudaStream_t stream;
+  bool own_stream;
+  eim::Comm* comm;
+  std::string last_error;
+  int sm_count;
+  uint64_t kernel_launches;
+
+  // arena (persistent, grows)
+  eim::DevBuf arena, set_start, set_len, covered;
+  eim::DevBuf ctl;            // SampleCtl
+  eim::DevBuf retry_a, retry_b;
+  eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
+  // per-graph vectors
+  eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
+  eim::DevBuf best, seeds, gains;
+  eim::DevBuf scratch;        // CUB temp storage
+  eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
+  void* h_pinned = nullptr;   // small pinned host scratch
+  cudaEvent_t ev0, ev1;
+};
+
+namespace eim {
+
+constexpr uint32_t CTX_MAGIC = 0xE1A0C7A7u;
+constexpr uint32_t GRAPH_MAGIC = 0xE1A06A7Fu;
+constexpr uint32_t SENTINEL = 0xFFFFFFFFu;
+
+// ---- graph.cu
+void graph_validate_and_thresholds(eim_ctx* ctx, eim_graph* g);
+
+// ---- sample.cu
+struct SampleResult {
+  uint64_t edges = 0;
+  uint64_t tier2 = 0;
+  uint32_t launches = 0;
+  double kernel_ms = 0;
+};
+// Samples ids [first, first+count) into ctx->arena; set index = id - set_base.
+// Histogram into C when hist is true.
+SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
+                          uint64_t first, uint64_t count, uint64_t set_base, bool hist);
+void arena_reset(eim_ctx* ctx);
+void ensure_sets(eim_ctx* ctx, uint64_t num_sets);
+uint64_t arena_cursor(eim_ctx* ctx);
+
+// ---- arena.cu
+// canonical export: offsets (count+1, device u64) + members (device u32), sets ascending
+uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members);
+// histogram of sets [lo, hi) into C_total
+void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi);
+// append externally supplied canonical sets (device pointers) as set ids [base, base+count)
+void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_offsets,
+                 const uint32_t* d_members, uint64_t total);
+
+// ---- select.cu
+// Greedy NodeSelection over sets [0, num_sets) with coverage C_total[0..n).
+// Writes seeds/gains (host), returns cov.
+uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
+                uint64_t* gains_out);
+
+// ---- imm.cpp
+void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);
+void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
+             uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
+             eim_stats* st);
+
+// ---- comm.cpp
+Comm* comm_create(int rank, int world, const void* id);
+void comm_destroy(Comm* c);
+void comm_get_id(void* out);
+void comm_allgather_u64(Comm* c, const uint64_t* d_send, uint64_t* d_recv, cudaStream_t st);
+void comm_broadcast(Comm* c, void* d_buf, size_t bytes, int root, cudaStream_t st);
+void comm_group_start();
+void comm_group_end();
+
+inline uint32_t grid_for(eim_ctx* ctx, uint64_t work, uint32_t per_block, uint32_t blocks_per_sm = 8) {
+  uint64_t b = (work + per_block - 1) / per_block;
+  uint64_t cap = (uint64_t)ctx->sm_count * blocks_per_sm;
+  if (b > cap) b = cap;
+  if (b == 0) b = 1;
+  return (uint32_t)b;
+}
+
+}  // namespace eim

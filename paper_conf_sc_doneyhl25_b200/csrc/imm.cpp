@@ -1,0 +1,180 @@
+// imm.cpp -- IMM driver (Alg. 1) with the martingale theta estimation
+// of [22] Alg. 2.  Scalars are host doubles (compiled with -ffp-contract=off,
+// evaluation order of reading R17); all data work is on the device.
+//
+// Multi-GPU (world > 1): each round's new sample ids [|R|, theta_i) are split
+// into contiguous shares (eim_shard_range), every rank samples its share,
+// the shares are all-gathered over NCCL in rank (= sample-id) order and the
+// greedy runs replicated on identical data, so results equal the 1-GPU run.
+#include <chrono>
+#include <cmath>
+#include <cstring>
+
+#include "eim_internal.h"
+
+namespace eim {
+
+uint64_t compact_range(eim_ctx* ctx, uint64_t lo, uint64_t count, uint64_t** d_offsets, uint32_t** d_members);
+
+void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* p) {
+  const double dn = (double)n;
+  const double ln_n = std::log(dn);
+  p->ell_p = ell * (1.0 + std::log(2.0) / ln_n);                 // [22] Alg. 1 l.1
+  p->eps_p = std::sqrt(2.0) * eps;                                // [22] Alg. 2
+  double lnC = 0.0;                                               // ln binom(n,k), in order
+  for (uint32_t i = 1; i <= k; ++i) lnC += std::log((double)(n - k + i)) - std::log((double)i);
+  p->lnC = lnC;
+  p->log2n = std::log2(dn);
+  p->lambda_p = (2.0 + (2.0 / 3.0) * p->eps_p) * (lnC + p->ell_p * ln_n + std::log(p->log2n)) * dn /
+                (p->eps_p * p->eps_p);                            // Eq. 9
+  const double e1 = 1.0 - 1.0 / std::exp(1.0);
+  const double alpha = std::sqrt(p->ell_p * ln_n + std::log(2.0));
+  const double beta = std::sqrt(e1 * (lnC + p->ell_p * ln_n + std::log(2.0)));
+  const double t = e1 * alpha + beta;
+  p->lambda_s = 2.0 * dn * (t * t) / (eps * eps);                 // Eq. 6
+}
+
+namespace {
+
+using clk = std::chrono::steady_clock;
+double ms_since(clk::time_point t0) {
+  return std::chrono::duration<double, std::milli>(clk::now() - t0).count();
+}
+
+struct Exchange {
+  DevBuf counts, offs_recv, mem_recv, len_send;
+};
+
+// Sample ids [R, R_new) across ranks; afterwards every rank holds all of them.
+void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t R, uint64_t R_new,
+                  eim_stats* st, Exchange& ex) {
+  const auto t0 = clk::now();
+  if (ctx->world == 1) {
+    SampleResult r = sample_range(ctx, g, model, seed, R, R_new - R, 0, true);
+    st->edges_examined += r.edges;
+    st->tier2_samples += r.tier2;
+    st->sample_launches += r.launches;
+    st->ms_sample_kernel += r.kernel_ms;
+    st->ms_sample += ms_since(t0);
+    return;
+  }
+  cudaStream_t s = ctx->stream;
+  uint64_t lo, hi;
+  eim_shard_range(R, R_new - R, ctx->rank, ctx->world, &lo, &hi);
+  SampleResult r = sample_range(ctx, g, model, seed, lo, hi - lo, 0, false);
+  st->edges_examined += r.edges;
+  st->tier2_samples += r.tier2;
+  st->sample_launches += r.launches;
+  st->ms_sample_kernel += r.kernel_ms;
+  const auto tc = clk::now();
+  ensure_sets(ctx, R_new);
+  // own share, compacted in sample-id order (offsets relative to the share)
+  uint64_t* d_off = nullptr;
+  uint32_t* d_mem = nullptr;
+  const uint64_t my_total = compact_range(ctx, lo, hi - lo, &d_off, &d_mem);
+  const int W = ctx->world;
+  ex.counts.reserve(2 * W * sizeof(uint64_t), false, s);
+  uint64_t* d_counts = ex.counts.as<uint64_t>();
+  EIM_CUDA(cudaMemcpyAsync(d_counts, &my_total, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+  comm_allgather_u64(ctx->comm, d_counts, d_counts + W, s);
+  std::vector<uint64_t> totals(W);
+  EIM_CUDA(cudaMemcpyAsync(totals.data(), d_counts + W, W * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  EIM_CUDA(cudaStreamSynchronize(s));
+  uint64_t max_total = 1, max_sets = 1;
+  for (int q = 0; q < W; ++q) {
+    uint64_t a, b;
+    eim_shard_range(R, R_new - R, q, W, &a, &b);
+    max_total = std::max(max_total, totals[q]);
+    max_sets = std::max(max_sets, b - a + 1);
+  }
+  ex.offs_recv.reserve(max_sets * sizeof(uint64_t), false, s);
+  ex.mem_recv.reserve(max_total * sizeof(uint32_t), false, s);
+  for (int q = 0; q < W; ++q) {
+    uint64_t a, b;
+    eim_shard_range(R, R_new - R, q, W, &a, &b);
+    if (b == a) continue;
+    uint64_t* offs = (q == ctx->rank) ? d_off : ex.offs_recv.as<uint64_t>();
+    uint32_t* mem = (q == ctx->rank) ? d_mem : ex.mem_recv.as<uint32_t>();
+    comm_group_start();
+    comm_broadcast(ctx->comm, offs, (b - a + 1) * sizeof(uint64_t), q, s);
+    if (totals[q]) comm_broadcast(ctx->comm, mem, totals[q] * sizeof(uint32_t), q, s);
+    comm_group_end();
+    if (q != ctx->rank) append_sets(ctx, a, b - a, offs, mem, totals[q]);
+  }
+  hist_sets(ctx, R, R_new);
+  EIM_CUDA(cudaStreamSynchronize(s));
+  st->ms_comm += ms_since(tc);
+  st->ms_sample += ms_since(t0);
+}
+
+}  // namespace
+
+void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
+             uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, eim_stats* st) {
+  const auto t_start = clk::now();
+  const uint32_t n = g->view.n;
+  eim_imm_params_t p;
+  imm_params(n, k, eps, ell, &p);
+  std::memset(st, 0, sizeof(*st));
+  st->lambda_p = p.lambda_p;
+  st->lambda_s = p.lambda_s;
+  const uint64_t launches0 = ctx->kernel_launches;
+  cudaStream_t s = ctx->stream;
+  // fresh arena + coverage for this graph
+  arena_reset(ctx);
+  ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
+  EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
+  Exchange ex;
+  std::vector<uint32_t> S(k);
+  uint64_t R = 0, cov = 0;
+  uint64_t R_selected = UINT64_MAX;  // |R| the last NodeSelection ran on
+  double LB = 1.0;
+  for (uint32_t i = 1; (double)i < p.log2n; ++i) {
+    const uint64_t theta_i = (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n);
+    if (theta_i > R) {
+      sample_round(ctx, g, model, seed, R, theta_i, st, ex);
+      R = theta_i;
+    }
+    const auto ts = clk::now();
+    cov = greedy(ctx, n, R, k, S.data(), nullptr);
+    st->ms_select += ms_since(ts);
+    R_selected = R;
+    if (st->rounds < 64) {
+      st->theta_i[st->rounds] = R;
+      st->cov_i[st->rounds] = cov;
+    }
+    st->rounds++;
+    if ((double)cov * std::ldexp(1.0, (int)i) >= (1.0 + p.eps_p) * (double)R) {
+      LB = ((double)n * (double)cov) / ((1.0 + p.eps_p) * (double)R);
+      break;
+    }
+  }
+  st->lb = LB;
+  const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
+  if (theta > R) {
+    sample_round(ctx, g, model, seed, R, theta, st, ex);
+    R = theta;
+  }
+  if (R != R_selected) {  // NodeSelection is deterministic: reuse the last run on the same R
+    const auto ts = clk::now();
+    cov = greedy(ctx, n, R, k, S.data(), nullptr);
+    st->ms_select += ms_since(ts);
+  }
+  std::memcpy(seeds_out, S.data(), (size_t)k * sizeof(uint32_t));
+  st->theta = R;
+  st->cov = cov;
+  st->arena_elems = 0;
+  {
+    // arena elements of all sets = sum of C_total
+    st->arena_elems = arena_cursor(ctx);
+  }
+  ex.counts.release();
+  ex.offs_recv.release();
+  ex.mem_recv.release();
+  if (theta_out) *theta_out = R;
+  if (spread_out) *spread_out = (double)n * (double)cov / (double)R;
+  st->kernel_launches = ctx->kernel_launches - launches0;
+  st->ms_total = ms_since(t_start);
+}
+
+}  // namespace eim

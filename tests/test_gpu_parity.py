@@ -1,0 +1,195 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE north_star): RRR sets, coverage, theta and seed sets
+bit-exact; spread (a double computed from the same integers) identical.
+Sizes span several tiles and ragged tails; the full-size configs run the
+launch configuration bench.py times (eim_imm_run on C2), with the oracle
+multi-threaded over sample ids (identical results by construction).
+"""
+import os
+
+import numpy as np
+import pytest
+
+import inputs
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+NT = max(1, min(64, os.cpu_count() or 1))
+
+
+@pytest.fixture(scope="module")
+def eim():
+    from paper_conf_sc_doneyhl25_b200 import _build
+    _build.build()
+    import paper_conf_sc_doneyhl25_b200 as E
+    return E
+
+
+@pytest.fixture(scope="module")
+def ctx(eim):
+    c = eim.eim_create(0)
+    yield c
+    eim.eim_destroy(c)
+
+
+@pytest.fixture(scope="module")
+def graphs():
+    cache = {}
+
+    def get(name):
+        if name not in cache:
+            cache[name] = inputs.config_graph(name)
+        return cache[name]
+    return get
+
+
+def _sets_equal(eim, ctx, g, off, nbr, model, seed, first, count):
+    go, gm = eim.eim_sample_rrr(ctx, g, model, seed, first, count)
+    ro, rm, _ = oracle.sample(off, nbr, model, seed, first, count, nthreads=NT)
+    assert np.array_equal(go, ro), (model, first, count)
+    assert np.array_equal(gm, rm), (model, first, count)
+    return ro
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_sample_rrr_C1_all_ids(eim, ctx, graphs, model):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        for seed in (1, 2, 3):
+            _sets_equal(eim, ctx, g, off, nbr, model, seed, 0, 30000)
+        # ragged tails, far ids, composability
+        _sets_equal(eim, ctx, g, off, nbr, model, 1, 2**40 + 17, 1)
+        _sets_equal(eim, ctx, g, off, nbr, model, 1, 2**61, 777)
+        a = eim.eim_sample_rrr(ctx, g, model, 5, 100, 33)
+        b = eim.eim_sample_rrr(ctx, g, model, 5, 133, 90)
+        c = eim.eim_sample_rrr(ctx, g, model, 5, 100, 123)
+        assert np.array_equal(np.concatenate([a[1], b[1]]), c[1])
+        o, m = eim.eim_sample_rrr(ctx, g, model, 5, 0, 0)
+        assert o.tolist() == [0] and m.size == 0
+    finally:
+        eim.eim_graph_free(g)
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+@pytest.mark.parametrize("shape", ["empty", "path", "star", "cycle", "bigcycle", "longpath", "rmat_dense"])
+def test_sample_rrr_special_graphs(eim, ctx, model, shape):
+    # bigcycle (every set = V, 3000 > tier-1 queue) and longpath force the
+    # global-memory tiers; rmat_dense has heavy rows and many live edges.
+    off, nbr = {
+        "empty": lambda: inputs.empty_graph(100),
+        "path": lambda: inputs.path_graph(50),
+        "star": lambda: inputs.star_out(70),
+        "cycle": lambda: inputs.cycle_graph(40),
+        "bigcycle": lambda: inputs.cycle_graph(3000),
+        "longpath": lambda: inputs.path_graph(5000),
+        "rmat_dense": lambda: inputs.rmat(600, 60000, seed=4),
+    }[shape]()
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        _sets_equal(eim, ctx, g, off, nbr, model, 9, 0, 700)
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_select_seeds_on_oracle_arenas(eim, ctx, graphs):
+    rng = np.random.default_rng(0)
+    for trial in range(30):
+        n = int(rng.integers(2, 300))
+        num = int(rng.integers(0, 500))
+        lens = rng.integers(1, min(n, 12) + 1, size=num)
+        offs = np.zeros(num + 1, dtype=np.uint64)
+        offs[1:] = np.cumsum(lens)
+        mem = np.concatenate([rng.choice(n, size=int(L), replace=False) for L in lens]).astype(np.uint32) \
+            if num else np.zeros(0, dtype=np.uint32)
+        k = int(rng.integers(1, n + 1))
+        s, gn = eim.eim_select_seeds(ctx, n, offs, mem, k)
+        rs, rg, _ = oracle.greedy(n, offs, mem, k)
+        assert np.array_equal(s, rs) and np.array_equal(gn, rg), trial
+    off, nbr = graphs("C1")
+    ro, rm, _ = oracle.sample(off, nbr, "IC", 3, 0, 5000, nthreads=NT)
+    s, gn = eim.eim_select_seeds(ctx, 1024, ro, rm, 40)
+    rs, rg, _ = oracle.greedy(1024, ro, rm, 40)
+    assert np.array_equal(s, rs) and np.array_equal(gn, rg)
+
+
+def _imm_equal(eim, ctx, g, off, nbr, k, eps, ell, model, seed):
+    seeds, theta, spread, st = eim.eim_imm_run(ctx, g, k, eps, ell, model, seed)
+    ref = oracle.imm(off, nbr, k, eps, ell, model, seed, nthreads=NT)
+    assert np.array_equal(seeds, ref["seeds"]), (model, seed)
+    assert theta == ref["theta"]
+    assert spread == ref["spread"]
+    assert st["theta_i"] == ref["theta_i"] and st["cov_i"] == ref["cov_i"]
+    assert st["lb"] == ref["lb"] and st["cov"] == ref["cov"]
+    assert st["lambda_p"] == ref["lambda_p"] and st["lambda_s"] == ref["lambda_s"]
+    assert st["edges_examined"] == ref["edges_examined"]
+    assert st["arena_elems"] == ref["arena_elems"]
+    return st
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_imm_C1(eim, ctx, graphs, model, seed):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        for k, eps in ((5, 0.5), (1, 0.9), (50, 0.2), (1024, 0.5)):
+            _imm_equal(eim, ctx, g, off, nbr, k, eps, 1.0, model, seed)
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_imm_degenerate_graphs(eim, ctx):
+    for off, nbr in (inputs.empty_graph(64), inputs.path_graph(32), inputs.cycle_graph(700), inputs.star_out(90)):
+        g = eim.eim_load_graph_csr(ctx, off, nbr)
+        try:
+            for model in ("IC", "LT"):
+                _imm_equal(eim, ctx, g, off, nbr, 3, 0.5, 1.0, model, 7)
+        finally:
+            eim.eim_graph_free(g)
+
+
+def test_invalid_graphs_rejected(eim, ctx):
+    off, nbr = inputs.path_graph(10)
+    bad_nbr = nbr.copy()
+    bad_nbr[3] = 10
+    bad_off = off.copy()
+    bad_off[4], bad_off[5] = bad_off[5], bad_off[4]
+    for o, m in ((off, bad_nbr), (bad_off, nbr)):
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_load_graph_csr(ctx, o, m)
+        assert ei.value.status == eim.EIM_E_INVAL
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    with pytest.raises(eim.EimError):
+        eim.eim_imm_run(ctx, g, 0, 0.5, 1.0, "IC", 1)
+    with pytest.raises(eim.EimError):
+        eim.eim_imm_run(ctx, g, 3, 1.5, 1.0, "IC", 1)
+    eim.eim_graph_free(g)
+    assert eim.lib().eim_graph_free(g) == eim.EIM_E_STATE
+
+
+# ---------------------------------------------------------------- full size
+def test_C2_sampled_sets_and_imm(eim, ctx, graphs):
+    c = inputs.CONFIGS["C2"]
+    off, nbr = graphs("C2")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 0, 3000)
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 98765, 1500)
+        st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
+        assert st["theta"] > 50000
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_C3_sampled_sets_and_imm(eim, ctx, graphs):
+    c = inputs.CONFIGS["C3"]
+    off, nbr = graphs("C3")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        _sets_equal(eim, ctx, g, off, nbr, "LT", 1, 0, 20000)
+        _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
+    finally:
+        eim.eim_graph_free(g)
