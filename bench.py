@@ -243,7 +243,7 @@ def main():
     off_p = torch.from_numpy(off).pin_memory()
     nbr_p = torch.from_numpy(nbr).pin_memory()
     e2e_ms = []
-    for i in range(args.e2e_steps + 1):
+    for i in range(args.e2e_steps + 1 if args.e2e_steps > 0 else 0):
         flush.zero_()
         barrier()
         t0 = time.perf_counter()
@@ -255,7 +255,7 @@ def main():
         if i > 0:
             e2e_ms.append(dt)
         assert np.array_equal(s2, seeds) and th2 == theta_all
-    te = torch.tensor([statistics.mean(e2e_ms)], dtype=torch.float64, device=dev)
+    te = torch.tensor([statistics.mean(e2e_ms) if e2e_ms else float("nan")], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_ms_step = float(te.item())
