@@ -87,6 +87,8 @@ struct eim_ctx {
   eim::DevBuf ctl;            // SampleCtl
   eim::DevBuf retry_a, retry_b;
   eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
+  eim::DevBuf table, rsizes, rfailed, rfill;    // per-round membership table + per-sample scratch
+  double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;

@@ -1,26 +1,28 @@
 // sample.cu -- RRR-set samplers (Alg. 2, P:107 for IC; P:134-140 for LT).
 //
-// IC, tier 1 (ic_tier1): one warp per sample id (ids handed out by a launch
-//   ticket).  The BFS queue Q and an open-addressing visited hash
-//   live in shared memory.  The frontier is expanded in batches of up to 32
-//   queued vertices: their in-rows are merged into one space of Philox quads
-//   (4 consecutive edge ids share one Philox4x32-10 call, reading R1), and
-//   the 32 lanes sweep that space, so small rows do not idle the warp and a
-//   hub row is split evenly.  An edge into u is live iff its draw <= T_u
-//   (R2).  in_nbr[e] is read only for live edges.  Newly visited vertices are
-//   appended with a warp ballot (no atomics on the queue tail).  A set that
-//   outgrows the shared-memory queue is abandoned and its id is pushed onto
-//   a retry list: the keyed randomness makes the redo exact.
-// IC, tier k >= 2 (ic_tierk): the same warp routine with the hash and queue
-//   in global memory (generation-tagged 64-bit slots, so no clearing), with
-//   capacities growing x16 per tier until they cover n.
-// LT, tier 1 (lt_tier1): one thread per reverse walk (the walk is
-//   sequential); the path lives in shared memory and is also the
-//   visited set.  Tier k: path + generation hash in global memory.
-// Every finished set reserves its arena range with one atomic (the arena is
-// append-only; set i is (set_start[i], set_len[i])) and bumps the coverage
-// histogram C (Alg. 2 l.25).  Member order inside a set is not canonical;
-// eim_sample_rrr sorts on export.
+// One sampler launch handles a contiguous range of sample ids [first,
+// first+count) (a "round").  Membership of every set of the round is kept in
+// ONE global open-addressing table keyed by (sample, vertex) (64-bit keys,
+// ~32 MB at C2, L2-resident), so no set ever outgrows its storage: the
+// per-sample state on chip is only the FRONTIER (discovered, not yet
+// expanded vertices).  After the launch the per-sample sizes are scanned into
+// arena offsets (sample-id order) and a scatter pass over the table writes
+// every member into the arena and bumps the coverage histogram C (Alg. 2 l.25)
+// -- placement is deterministic, no reservation atomics, no arena overflow.
+//
+// IC (ic_group_kernel<G, GLOBAL_RING>): G threads cooperate on one sample.  A
+//   batch of up to G frontier vertices has its in-rows merged into one space
+//   of Philox quads (4 consecutive edge ids share one Philox4x32-10 call,
+//   reading R1) that the G threads sweep, so small rows do not idle threads
+//   and hub rows split evenly.  An edge into u is live iff its draw <= T_u
+//   (R2); in_nbr[e] is read only for live edges.  Heavy samples under WC are
+//   chains of ~100 hub expansions, so G threads per sample (not a warp) keep
+//   the per-level latency low, and they start as soon as their id is drawn.
+//   The frontier lives in a shared-memory ring (tier 1); a sample whose
+//   backlog outgrows the ring is redone by a 512-thread group with the ring
+//   in global memory (tier 2, capacity n) under a distinct key tag.
+// LT (lt_kernel): one thread per reverse walk (sequential by nature),
+//   visited set = the same global table; no capacity limit.
 #include <cub/cub.cuh>
 
 #include "eim_internal.h"
@@ -31,58 +33,35 @@ namespace eim {
 namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
+constexpr uint32_t MAX_PROBE = 256;
 
-__device__ __forceinline__ uint32_t hash_slot(uint32_t v, uint32_t bits) {
-  return (v * 0x9E3779B1u) >> (32u - bits);
+// ---------------------------------------------------------------- table
+// key = ((s_local + 1) | tier << 31) << 32 | v ;  0 = empty slot.
+__device__ __forceinline__ unsigned long long table_key(uint32_t s_local, uint32_t tier, uint32_t v) {
+  return ((unsigned long long)((s_local + 1u) | (tier << 31)) << 32) | (unsigned long long)v;
 }
 
-// Shared-memory visited table: u32 slots holding v+1 (0 = empty).
-struct SmemTable {
-  uint32_t* h;
-  uint32_t bits;
-  __device__ __forceinline__ bool insert(uint32_t v) const {
-    const uint32_t key = v + 1u, mask = (1u << bits) - 1u;
-    uint32_t i = hash_slot(v, bits);
-    for (;;) {
-      uint32_t old = atomicCAS(&h[i], 0u, key);
-      if (old == 0u) return true;
-      if (old == key) return false;
-      i = (i + 1u) & mask;
-    }
-  }
-  __device__ __forceinline__ void clear(int lane) const {
-    uint4* p = reinterpret_cast<uint4*>(h);
-    for (uint32_t i = lane; i < (1u << bits) / 4u; i += 32u) p[i] = make_uint4(0, 0, 0, 0);
-  }
-};
+__device__ __forceinline__ uint32_t table_hash(unsigned long long key, uint32_t bits) {
+  unsigned long long h = key * 0x9E3779B97F4A7C15ull;
+  h ^= h >> 29;
+  h *= 0xBF58476D1CE4E5B9ull;
+  return (uint32_t)(h >> (64 - bits));
+}
 
-// Global-memory visited table: 64-bit slots (gen << 32 | v+1); a slot whose
-// generation differs from the current sample's is free.
-struct GenTable {
-  unsigned long long* h;
-  uint32_t bits;
-  uint32_t gen;
-  __device__ __forceinline__ bool insert(uint32_t v) const {
-    const unsigned long long want = ((unsigned long long)gen << 32) | (unsigned long long)(v + 1u);
-    const uint32_t mask = (1u << bits) - 1u;
-    uint32_t i = hash_slot(v, bits);
-    unsigned long long cur = __ldcg(&h[i]);
-    for (;;) {
-      if ((uint32_t)(cur >> 32) != gen) {
-        unsigned long long prev = atomicCAS(&h[i], cur, want);
-        if (prev == cur) return true;
-        cur = prev;
-        continue;
-      }
-      if (cur == want) return false;
-      i = (i + 1u) & mask;
-      cur = __ldcg(&h[i]);
-    }
+// 1 = inserted (new member), 0 = already present, -1 = table too full
+__device__ __forceinline__ int table_insert(unsigned long long* keys, uint32_t bits, unsigned long long key) {
+  const uint32_t mask = (uint32_t)((1ull << bits) - 1ull);
+  uint32_t i = table_hash(key, bits);
+  for (uint32_t p = 0; p < MAX_PROBE; ++p) {
+    const unsigned long long cur = atomicCAS(&keys[i], 0ull, key);
+    if (cur == 0ull) return 1;
+    if (cur == key) return 0;
+    i = (i + 1u) & mask;
   }
-};
+  return -1;
+}
 
-// Group barrier: a warp uses __syncwarp, larger groups a named barrier
-// (ids 1..15; id 0 is __syncthreads).
+// ---------------------------------------------------------------- groups
 template <int G>
 __device__ __forceinline__ void gsync(int gi) {
   if constexpr (G == 32) {
@@ -92,25 +71,22 @@ __device__ __forceinline__ void gsync(int gi) {
   }
 }
 
-// Per-group control block and frontier-batch row descriptors (shared memory).
 struct GroupCtl {
-  uint32_t tail, flag, gen, pad;
-  unsigned long long s, start;
+  uint32_t tail, flag, s_local, pad;
   uint32_t wsum[16];
-  uint32_t pad2[8];
 };
+
 template <int G>
 struct GroupRows {
   unsigned long long q0[G];  // first Philox quad of the row
   uint32_t qend[G];          // inclusive scan of quad counts
   uint32_t nq[G];            // quads of the row
   uint32_t T[G];             // IC threshold of the row's vertex
-  uint8_t wlo[G], whi[G];    // first / last valid word in the first / last quad
+  uint8_t wlo[G], whi[G];    // first valid word of the first quad, last valid word of the last quad
 };
 
 template <int G>
-__device__ __forceinline__ uint32_t group_incl_scan(uint32_t x, int gtid, int gi, GroupCtl& gc,
-                                                    uint32_t& total) {
+__device__ __forceinline__ uint32_t group_incl_scan(uint32_t x, int gtid, int gi, GroupCtl& gc, uint32_t& total) {
   const int lane = gtid & 31, w = gtid >> 5;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -135,35 +111,46 @@ __device__ __forceinline__ uint32_t group_incl_scan(uint32_t x, int gtid, int gi
   }
 }
 
-// One IC RRR set by a group of G threads (Alg. 2 l.5-20).  The queue Q is
-// also the member list.  Frontier batches of up to G queued vertices have
-// their rows merged into one quad space swept by the whole group; there is no
-// per-level barrier beyond one per batch.  Returns false when the set
-// outgrows qcap or (cap_quads > 0) the sample exceeds cap_quads Philox quads:
-// the caller then re-queues the id for a larger tier.
-template <int G, class Tab>
-__device__ __forceinline__ bool ic_group_sample(const GraphView& g, const PhiloxKey& K, uint64_t s,
-                                                const Tab& tab, uint32_t* queue, uint32_t qcap,
-                                                GroupRows<G>& rw, GroupCtl& gc, int gtid, int gi,
-                                                uint32_t cap_quads, unsigned long long& se) {
+enum : uint32_t { FLAG_RING = 1u, FLAG_TABLE = 2u };
+
+struct RoundView {
+  unsigned long long* keys;
+  uint32_t bits;
+  uint32_t* sizes;     // [count] members per sample (s_local)
+  uint8_t* failed;     // [count] 1 = tier-1 attempt abandoned (its tier-0 keys are ignored)
+  uint64_t base;       // sample id of s_local = 0
+};
+
+// One IC RRR set (Alg. 2 l.5-20) by a group of G threads.  ring = frontier
+// backlog of capacity W (W a power of two).  Returns the flag (0 = success);
+// size = number of members.
+template <int G>
+__device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const PhiloxKey& K, const RoundView& R,
+                                                    uint32_t s_local, uint32_t tier, uint32_t* ring, uint32_t W,
+                                                    GroupRows<G>& rw, GroupCtl& gc, int gtid, int gi,
+                                                    unsigned long long& se, uint32_t& size) {
+  const uint64_t s = R.base + s_local;
   if (gtid == 0) {
     const uint32_t root = draw_root(s, g.n, K);
-    tab.insert(root);
-    queue[0] = root;
+    const int r = table_insert(R.keys, R.bits, table_key(s_local, tier, root));
+    ring[0] = root;
     gc.tail = 1;
-    gc.flag = 0;
+    gc.flag = (r < 0) ? FLAG_TABLE : 0u;
   }
   gsync<G>(gi);
-  uint32_t head = 0, quads_done = 0;
+  uint32_t head = 0;
   se = 0;
   for (;;) {
     const uint32_t tail = *(volatile uint32_t*)&gc.tail;
     const uint32_t flag = *(volatile uint32_t*)&gc.flag;
-    if (flag || head >= tail) return flag == 0;
+    if (flag || head >= tail) {
+      size = tail;
+      return flag;
+    }
     const uint32_t nb = min((uint32_t)G, tail - head);
     uint32_t nq = 0;
     if (gtid < nb) {
-      const uint32_t u = queue[head + gtid];
+      const uint32_t u = ring[(head + gtid) & (W - 1)];
       const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
       if (e1 > e0) {
         nq = (uint32_t)(((e1 - 1) >> 2) - (e0 >> 2) + 1);
@@ -178,13 +165,8 @@ __device__ __forceinline__ bool ic_group_sample(const GraphView& g, const Philox
     uint32_t total;
     const uint32_t incl = group_incl_scan<G>(nq, gtid, gi, gc, total);
     if (gtid < nb) rw.qend[gtid] = incl;
+    head += nb;  // ring slots [old head, head) are free again: their rows are staged
     gsync<G>(gi);
-    head += nb;
-    quads_done += total;
-    if (cap_quads && quads_done > cap_quads) {
-      gsync<G>(gi);  // everyone is past the reads of this batch's control words
-      return false;
-    }
     int r = -1;
     uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0;
     unsigned long long q0_r = 0;
@@ -216,12 +198,13 @@ __device__ __forceinline__ bool ic_group_sample(const GraphView& g, const Philox
           const int i = __ffs(live) - 1;
           live &= live - 1;
           const uint32_t v = g.nbr[(q << 2) + i];
-          if (*(volatile uint32_t*)&gc.tail >= qcap) {
-            gc.flag = 1;
-          } else if (tab.insert(v)) {
+          const int ins = table_insert(R.keys, R.bits, table_key(s_local, tier, v));
+          if (ins > 0) {
             const uint32_t pos = atomicAdd(&gc.tail, 1u);
-            if (pos < qcap) queue[pos] = v;
-            else gc.flag = 1;
+            if (pos - head < W) ring[pos & (W - 1)] = v;
+            else atomicOr(&gc.flag, FLAG_RING);
+          } else if (ins < 0) {
+            atomicOr(&gc.flag, FLAG_TABLE);
           }
         }
       }
@@ -230,97 +213,51 @@ __device__ __forceinline__ bool ic_group_sample(const GraphView& g, const Philox
   }
 }
 
-// Group-cooperative IC sampler.  GLOBAL = false: hash + queue in shared
-// memory (tiers 1 and 2); GLOBAL = true: generation-tagged hash + queue in
-// global memory, one slot per group (last tiers, capacity up to n).
-template <int G, bool GLOBAL>
-__global__ void __launch_bounds__(512) ic_group_kernel(GraphView g, uint64_t seed, uint64_t first, uint64_t count,
-                                                       const unsigned long long* ids, ArenaView A, SampleCtl* ctl,
-                                                       unsigned long long* retry_out, uint32_t hbits, uint32_t qcap,
-                                                       uint32_t cap_quads, unsigned long long* gtabs,
-                                                       uint32_t* gqueues, uint32_t* gens) {
+// tier 1 (GLOBAL_RING = false): shared-memory ring of W entries per group,
+// over the contiguous ids [0, count).  tier 2 (GLOBAL_RING = true): ring of W
+// entries per group slot in global memory, over a list of failed ids.
+template <int G, bool GLOBAL_RING>
+__global__ void __launch_bounds__(G == 512 ? 512 : 256) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
+                                                                        uint64_t count,
+                                                                        const uint32_t* __restrict__ ids,
+                                                                        uint32_t W, SampleCtl* ctl,
+                                                                        uint32_t* retry_out, uint32_t* gring) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int gi = threadIdx.x / G, gtid = threadIdx.x % G;
-  const size_t tab_bytes = GLOBAL ? 0 : ((size_t)4 << hbits) + (size_t)4 * qcap;
-  unsigned char* base = smem_raw + (size_t)gi * (sizeof(GroupCtl) + sizeof(GroupRows<G>) + tab_bytes);
+  const size_t per_group = sizeof(GroupCtl) + sizeof(GroupRows<G>) + (GLOBAL_RING ? 0 : (size_t)4 * W);
+  unsigned char* base = smem_raw + (size_t)gi * per_group;
   GroupCtl& gc = *reinterpret_cast<GroupCtl*>(base);
   GroupRows<G>& rw = *reinterpret_cast<GroupRows<G>*>(base + sizeof(GroupCtl));
   const uint64_t slot = (uint64_t)blockIdx.x * (blockDim.x / G) + gi;
-  uint32_t* queue;
-  SmemTable stab{nullptr, hbits};
-  unsigned long long* gh = nullptr;
-  if constexpr (GLOBAL) {
-    gh = gtabs + (slot << hbits);
-    queue = gqueues + slot * (uint64_t)qcap;
-  } else {
-    stab.h = reinterpret_cast<uint32_t*>(base + sizeof(GroupCtl) + sizeof(GroupRows<G>));
-    queue = stab.h + (1u << hbits);
-    for (uint32_t i = gtid; i < (1u << hbits) / 4u; i += G) reinterpret_cast<uint4*>(stab.h)[i] = make_uint4(0, 0, 0, 0);
-  }
+  uint32_t* ring = GLOBAL_RING ? gring + slot * (uint64_t)W
+                               : reinterpret_cast<uint32_t*>(base + sizeof(GroupCtl) + sizeof(GroupRows<G>));
+  const uint32_t tier = GLOBAL_RING ? 1u : 0u;
   const PhiloxKey K = philox_key(seed);
   unsigned long long edges_acc = 0;
-  gsync<G>(gi);
   for (;;) {
     if (gtid == 0) {
-      gc.s = atomicAdd(&ctl->ticket, 1ull);
-      if constexpr (GLOBAL) {
-        uint32_t gen = gens[slot] + 1u;
-        if (gen == 0u) gen = 1u;
-        gens[slot] = gen;
-        gc.gen = gen;
-      }
+      const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
+      gc.s_local = t < count ? (ids ? ids[t] : (uint32_t)t) : 0xFFFFFFFFu;
     }
     gsync<G>(gi);
-    const unsigned long long t = gc.s;
-    if (t >= count) break;
-    const uint64_t s = ids ? ids[t] : first + t;
+    const uint32_t s_local = gc.s_local;
+    if (s_local == 0xFFFFFFFFu) break;
     unsigned long long se = 0;
-    bool ok;
-    if constexpr (GLOBAL) {
-      const uint32_t gen = gc.gen;
-      if (gen == 1u) {  // fresh (or wrapped) generation counter: clear this slot's table once
-        for (uint64_t i = gtid; i < (1ull << hbits); i += G) gh[i] = 0ull;
-        __threadfence_block();
-        gsync<G>(gi);
-      }
-      GenTable tab{gh, hbits, gen};
-      ok = ic_group_sample<G>(g, K, s, tab, queue, qcap, rw, gc, gtid, gi, cap_quads, se);
-    } else {
-      ok = ic_group_sample<G>(g, K, s, stab, queue, qcap, rw, gc, gtid, gi, cap_quads, se);
-    }
-    const uint32_t size = gc.tail;
+    uint32_t size = 0;
+    const uint32_t flag = ic_group_sample<G>(g, K, R, s_local, tier, ring, W, rw, gc, gtid, gi, se, size);
     if (gtid == 0) {
-      unsigned long long start = ~0ull;
-      if (ok) {
-        const unsigned long long st = atomicAdd(A.cursor, (unsigned long long)size);
-        if (st + size <= A.cap) {
-          start = st;
-          A.set_start[s - A.set_base] = st;
-          A.set_len[s - A.set_base] = size;
-          atomicMax(A.valid_end, st + size);
-        } else {
-          atomicAdd(&ctl->arena_fail, 1ull);
-        }
+      if (flag == 0) {
+        R.sizes[s_local] = size;
+      } else if (flag & FLAG_TABLE) {
+        atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);  // table too full: host redoes the round
+      } else {
+        R.failed[s_local] = 1;
+        retry_out[atomicAdd(&ctl->retry_count, 1ull)] = s_local;
       }
-      if (start == ~0ull) retry_out[atomicAdd(&ctl->retry_count, 1ull)] = s;
-      gc.start = start;
     }
-    gsync<G>(gi);
-    const unsigned long long start = gc.start;
-    if (start != ~0ull) {
-      for (uint32_t i = gtid; i < size; i += G) {
-        const uint32_t v = queue[i];
-        A.elems[start + i] = v;
-        if (A.C) atomicAdd(&A.C[v], 1u);
-      }
-      edges_acc += se;
-    }
-    if constexpr (!GLOBAL) {
-      for (uint32_t i = gtid; i < (1u << hbits) / 4u; i += G) reinterpret_cast<uint4*>(stab.h)[i] = make_uint4(0, 0, 0, 0);
-    }
+    if (flag == 0) edges_acc += se;
     gsync<G>(gi);
   }
-  // per-thread examined-edge sums
   for (int o = 16; o > 0; o >>= 1) edges_acc += __shfl_xor_sync(FULL, edges_acc, o);
   if ((threadIdx.x & 31) == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
@@ -328,149 +265,92 @@ __global__ void __launch_bounds__(512) ic_group_kernel(GraphView g, uint64_t see
 // ---------------------------------------------------------------- LT
 // Reverse LT walk (R3-R5): at u with d^-(u) > 0, tau_u is the
 // LT-tagged draw of u and the chosen in-neighbour is position
-// floor(tau * d / 2^32) of u's row (the prefix-scan choice under WC weights);
-// the walk stops when d^-(u) = 0 or the chosen vertex is already in the set.
-__device__ __forceinline__ uint32_t lt_next(const GraphView& g, const PhiloxKey& K, uint64_t s,
-                                            uint32_t u, bool& has) {
-  const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
-  if (e1 == e0) {
-    has = false;
-    return 0;
-  }
-  has = true;
-  const uint4 w = philox_at((uint64_t)(u >> 2), s, TAG_LT, K);
-  const uint32_t tau = word_of(w, u & 3u);
-  const unsigned long long j = __umul64hi((unsigned long long)tau << 32, e1 - e0);
-  return g.nbr[e0 + j];
-}
-
-__device__ __forceinline__ void lt_commit(const ArenaView& A, SampleCtl* ctl, unsigned long long* retry_out,
-                                          uint64_t s, bool ok, uint32_t L, const uint32_t* path,
-                                          uint32_t stride, unsigned long long steps,
-                                          unsigned long long& edges_acc) {
-  bool fail = !ok;
-  if (ok) {
-    unsigned long long start = atomicAdd(A.cursor, (unsigned long long)L);
-    if (start + L <= A.cap) {
-      for (uint32_t i = 0; i < L; ++i) {
-        uint32_t v = path[(size_t)i * stride];
-        A.elems[start + i] = v;
-        if (A.C) atomicAdd(&A.C[v], 1u);
-      }
-      A.set_start[s - A.set_base] = start;
-      A.set_len[s - A.set_base] = L;
-      atomicMax(A.valid_end, start + L);
-      edges_acc += steps;
-    } else {
-      fail = true;
-      atomicAdd(&ctl->arena_fail, 1ull);
-    }
-  }
-  if (fail) {
-    unsigned long long p = atomicAdd(&ctl->retry_count, 1ull);
-    retry_out[p] = s;
-  }
-}
-
-template <int P>
-__global__ void __launch_bounds__(128) lt_tier1_kernel(GraphView g, uint64_t seed, uint64_t first,
-                                                       uint64_t count, const unsigned long long* ids,
-                                                       ArenaView A, SampleCtl* ctl,
-                                                       unsigned long long* retry_out) {
-  extern __shared__ __align__(16) uint32_t path_smem[];
-  uint32_t* path = path_smem + threadIdx.x;  // [i * blockDim + tid]
-  const uint32_t stride = blockDim.x;
+// floor(tau * d / 2^32) of u's row (the prefix-scan choice under WC
+// weights); the walk stops when d^-(u) = 0 or the chosen vertex is already in
+// the set.  One thread per walk; visited set = the round table.
+__global__ void __launch_bounds__(256) lt_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
+                                                 SampleCtl* ctl) {
   const PhiloxKey K = philox_key(seed);
   unsigned long long edges_acc = 0;
   for (;;) {
     const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
     if (t >= count) break;
-    const uint64_t s = ids ? ids[t] : first + t;
+    const uint32_t s_local = (uint32_t)t;
+    const uint64_t s = R.base + s_local;
     uint32_t u = draw_root(s, g.n, K);
-    path[0] = u;
+    bool ok = table_insert(R.keys, R.bits, table_key(s_local, 0, u)) >= 0;
     uint32_t L = 1;
     unsigned long long steps = 0;
-    bool ok = true;
-    for (;;) {
-      bool has;
-      const uint32_t v = lt_next(g, K, s, u, has);
-      if (!has) break;
+    while (ok) {
+      const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
+      if (e1 == e0) break;
       ++steps;
-      bool seen = false;
-      for (uint32_t i = 0; i < L; ++i) seen |= (path[i * stride] == v);
-      if (seen) break;
-      if (L == P) {
-        ok = false;
-        break;
-      }
-      path[L * stride] = v;
+      const uint4 w = philox_at((uint64_t)(u >> 2), s, TAG_LT, K);
+      const uint32_t tau = word_of(w, u & 3u);
+      const unsigned long long j = __umul64hi((unsigned long long)tau << 32, e1 - e0);
+      const uint32_t v = g.nbr[e0 + j];
+      const int ins = table_insert(R.keys, R.bits, table_key(s_local, 0, v));
+      if (ins == 0) break;
+      if (ins < 0) ok = false;
       ++L;
       u = v;
     }
-    lt_commit(A, ctl, retry_out, s, ok, L, path, stride, steps, edges_acc);
-  }
-  if (edges_acc) atomicAdd(&ctl->edges, edges_acc);
-}
-
-__global__ void __launch_bounds__(128) lt_tierk_kernel(GraphView g, uint64_t seed, uint64_t count,
-                                                       const unsigned long long* ids, ArenaView A,
-                                                       SampleCtl* ctl, unsigned long long* retry_out,
-                                                       unsigned long long* tabs, uint32_t tbits,
-                                                       uint32_t* queues, uint32_t qcap, uint32_t* gens) {
-  const uint64_t slot = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  unsigned long long* h = tabs + (slot << tbits);
-  uint32_t* path = queues + slot * (uint64_t)qcap;
-  const PhiloxKey K = philox_key(seed);
-  unsigned long long edges_acc = 0;
-  for (;;) {
-    const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
-    if (t >= count) break;
-    const uint64_t s = ids[t];
-    uint32_t gen = gens[slot] + 1u;
-    if (gen == 0u) gen = 1u;
-    gens[slot] = gen;
-    if (gen == 1u)
-      for (uint64_t i = 0; i < (1ull << tbits); ++i) h[i] = 0ull;
-    GenTable tab{h, tbits, gen};
-    uint32_t u = draw_root(s, g.n, K);
-    tab.insert(u);
-    path[0] = u;
-    uint32_t L = 1;
-    unsigned long long steps = 0;
-    bool ok = true;
-    for (;;) {
-      bool has;
-      const uint32_t v = lt_next(g, K, s, u, has);
-      if (!has) break;
-      ++steps;
-      if (!tab.insert(v)) break;
-      if (L == qcap) {
-        ok = false;
-        break;
-      }
-      path[L++] = v;
-      u = v;
+    if (ok) {
+      R.sizes[s_local] = L;
+      edges_acc += steps;
+    } else {
+      atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);
     }
-    lt_commit(A, ctl, retry_out, s, ok, L, path, 1, steps, edges_acc);
   }
   if (edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
 
-constexpr int LT_P = 64;                          // path capacity per walker (tier 1)
-constexpr int LT_THREADS = 128;
+// ---------------------------------------------------------------- output
+__global__ void sizes_to_offsets_kernel(const uint32_t* __restrict__ sizes, uint64_t count,
+                                        uint64_t* __restrict__ out) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= count; i += stride)
+    out[i] = i < count ? (uint64_t)sizes[i] : 0ull;
+}
 
-// IC tier table: group size, groups per block, log2 hash slots, queue capacity, work cap.
-struct IcTier {
-  int G, NG;
-  uint32_t hbits, qcap, cap_quads;
-  bool global;
-};
-constexpr IcTier IC_T1{32, 8, 9, 256, 2048, false};     // warp per sample, light samples
-constexpr IcTier IC_T2{128, 4, 12, 2048, 0, false};     // 4 warps per sample, heavy samples
+__global__ void place_sets_kernel(const uint64_t* __restrict__ excl, const uint32_t* __restrict__ sizes,
+                                  uint64_t count, uint64_t arena_base, uint64_t set_index0,
+                                  uint64_t* __restrict__ set_start, uint32_t* __restrict__ set_len) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
+    set_start[set_index0 + i] = arena_base + excl[i];
+    set_len[set_index0 + i] = sizes[i];
+  }
+}
 
-template <int G, bool GLOBAL>
-size_t ic_smem_per_group(uint32_t hbits, uint32_t qcap) {
-  return sizeof(GroupCtl) + sizeof(GroupRows<G>) + (GLOBAL ? 0 : ((size_t)4 << hbits) + (size_t)4 * qcap);
+// Every live table entry is a member: arena[start(s) + fill[s]++] = v.
+__global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint64_t nslots,
+                               const uint8_t* __restrict__ failed, const uint64_t* __restrict__ set_start,
+                               uint64_t set_index0, uint32_t* __restrict__ fill, uint32_t* __restrict__ arena,
+                               uint32_t* __restrict__ C) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nslots; i += stride) {
+    const unsigned long long k = keys[i];
+    if (k == 0ull) continue;
+    const uint32_t hi = (uint32_t)(k >> 32);
+    const uint32_t tier = hi >> 31;
+    const uint32_t s_local = (hi & 0x7FFFFFFFu) - 1u;
+    if (tier == 0 && failed[s_local]) continue;  // abandoned tier-1 attempt; redone under tier-2 keys
+    const uint32_t v = (uint32_t)k;
+    const uint32_t p = atomicAdd(&fill[s_local], 1u);
+    arena[set_start[set_index0 + s_local] + p] = v;
+    if (C) atomicAdd(&C[v], 1u);
+  }
+}
+
+constexpr int IC_G = 128;          // threads per sample, tier 1
+constexpr int IC_NG = 2;           // groups per block
+constexpr uint32_t IC_W = 1024;    // shared-memory frontier ring per group
+constexpr int IC_G2 = 512;         // tier 2 (global ring of capacity >= n)
+
+template <int G, bool GR>
+size_t ic_smem_per_group(uint32_t W) {
+  return sizeof(GroupCtl) + sizeof(GroupRows<G>) + (GR ? 0 : (size_t)4 * W);
 }
 
 }  // namespace
@@ -481,6 +361,7 @@ void arena_reset(eim_ctx* ctx) {
   ctx->ctl.reserve(sizeof(SampleCtl) + 2 * sizeof(unsigned long long), false, ctx->stream);
   // ctl layout: [SampleCtl][cursor][valid_end]
   EIM_CUDA(cudaMemsetAsync(ctx->ctl.p, 0, sizeof(SampleCtl) + 2 * sizeof(unsigned long long), ctx->stream));
+  ctx->est_mean_size = 0;
 }
 
 uint64_t arena_cursor(eim_ctx* ctx) {
@@ -496,27 +377,12 @@ void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
   ctx->set_len.reserve(num_sets * sizeof(uint32_t), true, ctx->stream);
 }
 
-static ArenaView arena_view(eim_ctx* ctx, uint64_t set_base, bool hist) {
-  ArenaView A;
-  unsigned long long* tail = reinterpret_cast<unsigned long long*>(ctx->ctl.as<SampleCtl>() + 1);
-  A.elems = ctx->arena.as<uint32_t>();
-  A.cursor = tail;
-  A.valid_end = tail + 1;
-  A.cap = ctx->arena.bytes / sizeof(uint32_t);
-  A.set_start = ctx->set_start.as<uint64_t>();
-  A.set_len = ctx->set_len.as<uint32_t>();
-  A.set_base = set_base;
-  A.C = hist ? ctx->C_total.as<uint32_t>() : nullptr;
-  return A;
-}
-
-template <int G, bool GLOBAL>
-static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, uint64_t first, uint64_t count,
-                      const unsigned long long* ids, const ArenaView& A, SampleCtl* ctl,
-                      unsigned long long* retry_out, uint32_t hbits, uint32_t qcap, uint32_t cap, int NG,
-                      uint64_t max_groups) {
-  const size_t smem = ic_smem_per_group<G, GLOBAL>(hbits, qcap) * NG;
-  auto kern = ic_group_kernel<G, GLOBAL>;
+template <int G, bool GR>
+static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, const RoundView& R, uint64_t count,
+                      const uint32_t* ids, uint32_t W, SampleCtl* ctl, uint32_t* retry_out, uint32_t* gring,
+                      int NG, uint64_t max_groups) {
+  const size_t smem = ic_smem_per_group<G, GR>(W) * NG;
+  auto kern = ic_group_kernel<G, GR>;
   EIM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, G * NG, smem));
@@ -525,11 +391,7 @@ static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, uint64_t 
   blocks = std::min<uint64_t>(blocks, (count + NG - 1) / NG);
   blocks = std::min<uint64_t>(blocks, std::max<uint64_t>(1, max_groups / NG));
   blocks = std::max<uint64_t>(blocks, 1);
-  unsigned long long* tabs = GLOBAL ? ctx->tier_tab.as<unsigned long long>() : nullptr;
-  uint32_t* queues = GLOBAL ? ctx->tier_queue.as<uint32_t>() : nullptr;
-  uint32_t* gens = GLOBAL ? ctx->tier_gen.as<uint32_t>() : nullptr;
-  kern<<<(uint32_t)blocks, G * NG, smem, ctx->stream>>>(g->view, seed, first, count, ids, A, ctl, retry_out, hbits,
-                                                         qcap, cap, tabs, queues, gens);
+  kern<<<(uint32_t)blocks, G * NG, smem, ctx->stream>>>(g->view, seed, R, count, ids, W, ctl, retry_out, gring);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
 }
@@ -538,105 +400,109 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
                           uint64_t first, uint64_t count, uint64_t set_base, bool hist) {
   SampleResult res;
   if (count == 0) return res;
+  if (count >= 0x7FFFFFF0ull) fail(EIM_E_INVAL, "at most 2^31 sets per sampler launch");
   cudaStream_t st = ctx->stream;
   ensure_sets(ctx, first + count - set_base);
-  ctx->retry_a.reserve(count * sizeof(unsigned long long), false, st);
-  ctx->retry_b.reserve(count * sizeof(unsigned long long), false, st);
   SampleCtl* ctl = ctx->ctl.as<SampleCtl>();
-  unsigned long long* tail = reinterpret_cast<unsigned long long*>(ctl + 1);
+  unsigned long long* d_cursor = reinterpret_cast<unsigned long long*>(ctl + 1);
   SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
-  unsigned long long* h_tail = reinterpret_cast<unsigned long long*>(h + 1);
-  unsigned long long* retry_in = ctx->retry_a.as<unsigned long long>();
-  unsigned long long* retry_out = ctx->retry_b.as<unsigned long long>();
-  uint32_t nbits = 1;
-  while ((1ull << nbits) < (uint64_t)g->view.n) nbits++;
+  unsigned long long* h_cursor = reinterpret_cast<unsigned long long*>(h + 1);
+  ctx->rsizes.reserve(count * sizeof(uint32_t), false, st);
+  ctx->rfailed.reserve(count, false, st);
+  ctx->rfill.reserve(count * sizeof(uint32_t), false, st);
+  ctx->retry_a.reserve(count * sizeof(uint32_t), false, st);
+  ctx->stage_a.reserve((count + 1) * sizeof(uint64_t), false, st);
 
-  auto read_ctl = [&]() {
+  // table capacity: >= 4x the expected members of the round (mean set size
+  // of earlier rounds, else 64), at least 2^20 slots
+  const double mean = ctx->est_mean_size > 0 ? ctx->est_mean_size : 64.0;
+  uint32_t bits = 20;
+  while (bits < 32 && (double)(1ull << bits) < 4.0 * mean * (double)count) bits++;
+
+  for (int attempt = 0;; ++attempt) {
+    ctx->table.reserve((8ull << bits), false, st);
+    RoundView R{ctx->table.as<unsigned long long>(), bits, ctx->rsizes.as<uint32_t>(), ctx->rfailed.as<uint8_t>(),
+                first};
+    EIM_CUDA(cudaMemsetAsync(R.keys, 0, 8ull << bits, st));
+    EIM_CUDA(cudaMemsetAsync(R.failed, 0, count, st));
+    EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
+    EIM_CUDA(cudaEventRecord(ctx->ev0, st));
+    if (model == EIM_IC) {
+      launch_ic<IC_G, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr,
+                             IC_NG, ~0ull);
+    } else {
+      int per_sm = 0;
+      EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel, 256, 0));
+      uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (count + 255) / 256);
+      lt_kernel<<<(uint32_t)blocks, 256, 0, st>>>(g->view, seed, R, count, ctl);
+      EIM_CUDA(cudaGetLastError());
+      ctx->kernel_launches++;
+    }
+    EIM_CUDA(cudaEventRecord(ctx->ev1, st));
     EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl) + 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     EIM_CUDA(cudaStreamSynchronize(st));
-    res.edges += h->edges;
-  };
-  auto grow_if_needed = [&]() {
-    if (!h->arena_fail) return;
-    // successful reservations form a prefix [0, valid_end): keep it, grow, rewind the cursor
-    const uint64_t valid = h_tail[1];
-    const uint64_t cap = ctx->arena.bytes / sizeof(uint32_t);
-    const uint64_t want = std::max<uint64_t>(cap * 2, valid * 2 + 4096ull * h->retry_count);
-    ctx->arena.reserve(want * sizeof(uint32_t), true, st);
-    EIM_CUDA(cudaMemcpyAsync(tail, &h_tail[1], sizeof(unsigned long long), cudaMemcpyHostToDevice, st));
-  };
-
-  // ---- tier 1 over the contiguous id range
-  EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
-  ArenaView A = arena_view(ctx, set_base, hist);
-  EIM_CUDA(cudaEventRecord(ctx->ev0, st));
-  if (model == EIM_IC) {
-    launch_ic<32, false>(ctx, g, seed, first, count, nullptr, A, ctl, retry_out, IC_T1.hbits, IC_T1.qcap,
-                         IC_T1.cap_quads, IC_T1.NG, ~0ull);
-  } else {
-    const size_t smem = (size_t)LT_P * LT_THREADS * sizeof(uint32_t);
-    int per_sm = 0;
-    EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_tier1_kernel<LT_P>, LT_THREADS, smem));
-    uint64_t blocks = (uint64_t)std::max(1, per_sm) * ctx->sm_count;
-    blocks = std::min<uint64_t>(blocks, (count + LT_THREADS - 1) / LT_THREADS);
-    lt_tier1_kernel<LT_P><<<(uint32_t)blocks, LT_THREADS, smem, st>>>(g->view, seed, first, count, nullptr, A, ctl,
-                                                                      retry_out);
-    EIM_CUDA(cudaGetLastError());
-    ctx->kernel_launches++;
-  }
-  EIM_CUDA(cudaEventRecord(ctx->ev1, st));
-  res.launches = 1;
-  read_ctl();
-  float ms = 0;
-  EIM_CUDA(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
-  res.kernel_ms = ms;
-
-  // ---- retry tiers over the re-queued ids
-  int tier = 1;
-  uint32_t qbits = (model == EIM_IC) ? 8 : 6;  // log2 capacity of the tier that failed
-  while (h->retry_count > 0) {
-    const uint64_t nretry = h->retry_count;
-    res.tier2 += nretry;
-    grow_if_needed();
-    std::swap(retry_in, retry_out);
-    EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
-    A = arena_view(ctx, set_base, hist);
-    ++tier;
-    if (model == EIM_IC && tier == 2) {
-      launch_ic<128, false>(ctx, g, seed, 0, nretry, retry_in, A, ctl, retry_out, IC_T2.hbits, IC_T2.qcap,
-                            IC_T2.cap_quads, IC_T2.NG, ~0ull);
-      qbits = 11;
-    } else {
-      // global-memory tiers: capacity x16 per tier until it covers n
-      qbits = std::min(std::max(qbits + 4, 16u), nbits);
-      const uint64_t qcap = 1ull << qbits;
-      const uint32_t tbits = qbits + 1;
-      const uint64_t per_slot = (8ull << tbits) + 4ull * qcap;
-      const uint64_t budget = 1ull << 30;
-      uint64_t slots = std::min<uint64_t>(nretry, std::max<uint64_t>(1, budget / per_slot));
-      slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count * (model == EIM_IC ? 2 : 64));
-      ctx->tier_tab.reserve(slots * (8ull << tbits), false, st);
-      ctx->tier_queue.reserve(slots * qcap * 4, false, st);
-      ctx->tier_gen.reserve(slots * 4, false, st);
-      EIM_CUDA(cudaMemsetAsync(ctx->tier_gen.p, 0, slots * 4, st));
-      if (model == EIM_IC) {
-        launch_ic<512, true>(ctx, g, seed, 0, nretry, retry_in, A, ctl, retry_out, tbits, (uint32_t)qcap, 0, 1, slots);
-      } else {
-        const uint32_t group = (uint32_t)std::min<uint64_t>(128, slots);
-        const uint32_t blocks = (uint32_t)((slots + group - 1) / group);
-        lt_tierk_kernel<<<blocks, group, 0, st>>>(g->view, seed, nretry, retry_in, A, ctl, retry_out,
-                                                  ctx->tier_tab.as<unsigned long long>(), tbits,
-                                                  ctx->tier_queue.as<uint32_t>(), (uint32_t)qcap,
-                                                  ctx->tier_gen.as<uint32_t>());
-        EIM_CUDA(cudaGetLastError());
-        ctx->kernel_launches++;
-      }
+    float ms = 0;
+    EIM_CUDA(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
+    res.kernel_ms += ms;
+    res.launches++;
+    uint64_t edges = h->edges;
+    bool table_full = h->arena_fail != 0;
+    if (!table_full && h->retry_count > 0) {
+      // tier 2: frontier backlog outgrew the shared ring; redo with a global ring of capacity >= n
+      const uint64_t nretry = h->retry_count;
+      res.tier2 += nretry;
+      uint32_t W2 = 1;
+      while (W2 < g->view.n) W2 <<= 1;
+      uint64_t slots = std::min<uint64_t>(nretry, std::max<uint64_t>(1, (1ull << 30) / (4ull * W2)));
+      slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count);
+      ctx->tier_queue.reserve(slots * (uint64_t)W2 * 4, false, st);
+      EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
+      launch_ic<IC_G2, true>(ctx, g, seed, R, nretry, ctx->retry_a.as<uint32_t>(), W2, ctl, nullptr,
+                             ctx->tier_queue.as<uint32_t>(), 1, slots);
+      EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
+      EIM_CUDA(cudaStreamSynchronize(st));
+      edges += h->edges;
+      table_full = h->arena_fail != 0;
+      if (!table_full && h->retry_count) fail(EIM_E_CUDA, "tier-2 sampler failed with a ring of capacity n");
     }
-    read_ctl();
-    if (h->retry_count == nretry && !h->arena_fail && qbits >= nbits && tier > 3)
-      fail(EIM_E_CUDA, "sampler made no progress at full capacity");
+    if (table_full) {
+      if (attempt >= 4 || bits >= 31) fail(EIM_E_NOMEM, "membership table overflow");
+      bits += 2;  // rare: redo the whole round with a 4x larger table
+      continue;
+    }
+    res.edges += edges;
+    // ---- sizes -> offsets (sample-id order) -> arena placement -> scatter + histogram
+    uint64_t* excl = ctx->stage_a.as<uint64_t>();
+    sizes_to_offsets_kernel<<<grid_for(ctx, count + 1, 256), 256, 0, st>>>(ctx->rsizes.as<uint32_t>(), count, excl);
+    EIM_CUDA(cudaGetLastError());
+    size_t tmp = 0;
+    EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, count + 1, st));
+    ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+    EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, count + 1, st));
+    EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + count, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    EIM_CUDA(cudaMemcpyAsync(h_cursor, d_cursor, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    EIM_CUDA(cudaStreamSynchronize(st));
+    const uint64_t total = h->ticket, cursor = h_cursor[0];
+    ctx->arena.reserve((cursor + total) * sizeof(uint32_t), true, st);
+    const uint64_t set_index0 = first - set_base;
+    place_sets_kernel<<<grid_for(ctx, count, 256), 256, 0, st>>>(excl, ctx->rsizes.as<uint32_t>(), count, cursor,
+                                                                  set_index0, ctx->set_start.as<uint64_t>(),
+                                                                  ctx->set_len.as<uint32_t>());
+    EIM_CUDA(cudaGetLastError());
+    EIM_CUDA(cudaMemsetAsync(ctx->rfill.p, 0, count * sizeof(uint32_t), st));
+    const uint64_t nslots = 1ull << bits;
+    scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
+        R.keys, nslots, R.failed, ctx->set_start.as<uint64_t>(), set_index0, ctx->rfill.as<uint32_t>(),
+        ctx->arena.as<uint32_t>(), hist ? ctx->C_total.as<uint32_t>() : nullptr);
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches += 5;
+    h_cursor[0] = cursor + total;
+    h_cursor[1] = cursor + total;
+    EIM_CUDA(cudaMemcpyAsync(d_cursor, h_cursor, 2 * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+    EIM_CUDA(cudaStreamSynchronize(st));
+    ctx->est_mean_size = std::max(1.0, (double)total / (double)count);
+    return res;
   }
-  return res;
 }
 
 }  // namespace eim

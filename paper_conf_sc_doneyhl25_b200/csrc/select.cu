@@ -101,27 +101,20 @@ __global__ void cover_kernel(uint32_t j, const unsigned long long* __restrict__ 
     gains[j] = key >> 32;
     if (j > 0) W[seeds[j - 1]] = SENTINEL;  // its sets are all covered: nobody else touches it
   }
+  // one warp per entry of v's inverted list: the covered sets are
+  // decremented in parallel across the whole grid
   const int lane = threadIdx.x & 31;
   const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   const uint64_t lo = inv_off[v], hi = inv_off[v + 1];
-  for (uint64_t p = lo + warp * 32; p < hi; p += nwarps * 32) {
-    uint32_t i = 0;
-    bool fresh = false;
-    if (p + lane < hi) {
-      i = inv[p + lane];
-      fresh = F[i] == 0;
-      if (fresh) F[i] = 1;  // set ids are unique within v's list: no race
-    }
-    unsigned bal = __ballot_sync(FULL, fresh);
-    while (bal) {
-      const int src = __ffs(bal) - 1;
-      bal &= bal - 1;
-      const uint32_t si = __shfl_sync(FULL, i, src);
-      const uint64_t st = set_start[si];
-      const uint32_t L = set_len[si];
-      for (uint32_t t = lane; t < L; t += 32) atomicSub(&W[arena[st + t]], 1u);
-    }
+  for (uint64_t p = lo + warp; p < hi; p += nwarps) {
+    const uint32_t i = inv[p];
+    if (F[i]) continue;  // covered by an earlier pick (set ids are unique within v's list)
+    __syncwarp();
+    if (lane == 0) F[i] = 1;
+    const uint64_t st = set_start[i];
+    const uint32_t L = set_len[i];
+    for (uint32_t t = lane; t < L; t += 32) atomicSub(&W[arena[st + t]], 1u);
   }
 }
 
@@ -167,7 +160,7 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   const uint32_t n4 = n_pad / 4;
   constexpr int AB = 256;
   const uint32_t ablocks = grid_for(ctx, n4, AB, 8);
-  const uint32_t cblocks = (uint32_t)ctx->sm_count * 2;
+  const uint32_t cblocks = (uint32_t)ctx->sm_count * 8;
   for (uint32_t j = 0; j < k; ++j) {
     argmax_kernel<AB><<<ablocks, AB, 0, st>>>(reinterpret_cast<const uint4*>(W), n4, ctx->seeds.as<uint32_t>(), j,
                                               ctx->best.as<unsigned long long>());
