@@ -281,7 +281,7 @@ def main():
                          "sample_kernel": k_ms / args.steps,
                          "select": sum(s["ms_select"] for s in stats) / args.steps,
                          "comm": sum(s["ms_comm"] for s in stats) / args.steps},
-            "roofline": {"bound": "alu", "kernel": "ic_tier1_kernel", "achieved": achieved, "peak": peak,
+            "roofline": {"bound": "alu", "kernel": "ic_group_kernel (all tiers)", "achieved": achieved, "peak": peak,
                          "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
                          "peak_basis": f"Philox issue roof: 148 SM x 4 sched x 32 lanes x {sm_max:.0f} MHz / 10 instr per edge (DESIGN.md §6)"},
             "cpu_baseline": cb,

@@ -9,7 +9,6 @@ namespace eim {
 
 namespace {
 
-constexpr unsigned FULL = 0xFFFFFFFFu;
 
 // One warp per set: C[x] += 1 for every member x (sets have no duplicates).
 __global__ void hist_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,

@@ -91,7 +91,8 @@ void free_ctx_buffers(eim_ctx* c) {
   DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->retry_a, &c->retry_b,
                     &c->tier_tab, &c->tier_queue, &c->tier_gen, &c->C_total, &c->C_work, &c->inv_off,
                     &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
-                    &c->stage_b, &c->stage_c, &c->table, &c->rsizes, &c->rfailed, &c->rfill};
+                    &c->stage_b, &c->stage_c, &c->table, &c->rsizes, &c->rfailed, &c->rfill,
+                    &c->cand, &c->cidx, &c->arena_c, &c->selected};
   for (DevBuf* b : bufs) b->release();
 }
 

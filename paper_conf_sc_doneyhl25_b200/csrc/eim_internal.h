@@ -92,6 +92,7 @@ struct eim_ctx {
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;
+  eim::DevBuf cand, cidx, arena_c, selected;  // greedy: candidates, remapped arena, picked flags
   eim::DevBuf scratch;        // CUB temp storage
   eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
   void* h_pinned = nullptr;   // small pinned host scratch

@@ -34,6 +34,9 @@ namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr uint32_t MAX_PROBE = 256;
+constexpr int IC_G = 256;          // threads per sample (one block), tier 1
+constexpr int IC_NG = 1;           // groups per block
+constexpr int IC_U = 2;            // quads per thread per sweep iteration
 
 // ---------------------------------------------------------------- table
 // key = ((s_local + 1) | tier << 31) << 32 | v ;  0 = empty slot.
@@ -62,13 +65,10 @@ __device__ __forceinline__ int table_insert(unsigned long long* keys, uint32_t b
 }
 
 // ---------------------------------------------------------------- groups
+// One group = one block (G = blockDim.x), so a group barrier is __syncthreads.
 template <int G>
-__device__ __forceinline__ void gsync(int gi) {
-  if constexpr (G == 32) {
-    __syncwarp();
-  } else {
-    asm volatile("bar.sync %0, %1;" ::"r"(gi + 1), "r"(G) : "memory");
-  }
+__device__ __forceinline__ void gsync(int) {
+  __syncthreads();
 }
 
 struct GroupCtl {
@@ -124,7 +124,7 @@ struct RoundView {
 // One IC RRR set (Alg. 2 l.5-20) by a group of G threads.  ring = frontier
 // backlog of capacity W (W a power of two).  Returns the flag (0 = success);
 // size = number of members.
-template <int G>
+template <int G, int U>
 __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const PhiloxKey& K, const RoundView& R,
                                                     uint32_t s_local, uint32_t tier, uint32_t* ring, uint32_t W,
                                                     GroupRows<G>& rw, GroupCtl& gc, int gtid, int gi,
@@ -167,37 +167,55 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
     if (gtid < nb) rw.qend[gtid] = incl;
     head += nb;  // ring slots [old head, head) are free again: their rows are staged
     gsync<G>(gi);
+    // Sweep the batch's quad space; each thread takes U quads per iteration
+    // (j, j+G, .., j+(U-1)G) whose Philox chains are independent (ILP).
     int r = -1;
     uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0;
     unsigned long long q0_r = 0;
-    for (uint32_t base = 0; base < total; base += G) {
-      const uint32_t j = base + gtid;
-      if (j < total) {
-        if (j >= qe) {
-          do {
-            ++r;
-            qe = rw.qend[r];
-          } while (j >= qe);
-          nq_r = rw.nq[r];
-          qb = qe - nq_r;
-          q0_r = rw.q0[r];
-          T_r = rw.T[r];
-          wlo_r = rw.wlo[r];
-          whi_r = rw.whi[r];
+    for (uint32_t base = 0; base < total; base += U * G) {
+      unsigned long long qk[U];
+      uint32_t Tk[U], mk[U];
+#pragma unroll
+      for (int k = 0; k < U; ++k) {
+        const uint32_t j = base + k * G + gtid;
+        mk[k] = 0u;
+        qk[k] = 0ull;
+        Tk[k] = 0u;
+        if (j < total) {
+          if (j >= qe) {
+            do {
+              ++r;
+              qe = rw.qend[r];
+            } while (j >= qe);
+            nq_r = rw.nq[r];
+            qb = qe - nq_r;
+            q0_r = rw.q0[r];
+            T_r = rw.T[r];
+            wlo_r = rw.wlo[r];
+            whi_r = rw.whi[r];
+          }
+          const uint32_t li = j - qb;
+          uint32_t m = 0xFu;
+          if (li == 0) m &= 0xFu << wlo_r;
+          if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
+          mk[k] = m;
+          qk[k] = q0_r + li;
+          Tk[k] = T_r;
         }
-        const uint32_t li = j - qb;
-        const unsigned long long q = q0_r + li;
-        const uint4 w = philox_at(q, s, TAG_EDGE, K);
-        uint32_t m = 0xFu;
-        if (li == 0) m &= 0xFu << wlo_r;
-        if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
-        uint32_t live = (w.x <= T_r ? 1u : 0u) | (w.y <= T_r ? 2u : 0u) | (w.z <= T_r ? 4u : 0u) |
-                        (w.w <= T_r ? 8u : 0u);
-        live &= m;
+      }
+      uint4 wk[U];
+#pragma unroll
+      for (int k = 0; k < U; ++k) wk[k] = philox_at(qk[k], s, TAG_EDGE, K);
+#pragma unroll
+      for (int k = 0; k < U; ++k) {
+        const uint32_t T = Tk[k];
+        uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
+                        (wk[k].w <= T ? 8u : 0u);
+        live &= mk[k];
         while (live) {
           const int i = __ffs(live) - 1;
           live &= live - 1;
-          const uint32_t v = g.nbr[(q << 2) + i];
+          const uint32_t v = g.nbr[(qk[k] << 2) + i];
           const int ins = table_insert(R.keys, R.bits, table_key(s_local, tier, v));
           if (ins > 0) {
             const uint32_t pos = atomicAdd(&gc.tail, 1u);
@@ -217,7 +235,7 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
 // over the contiguous ids [0, count).  tier 2 (GLOBAL_RING = true): ring of W
 // entries per group slot in global memory, over a list of failed ids.
 template <int G, bool GLOBAL_RING>
-__global__ void __launch_bounds__(G == 512 ? 512 : 256) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
+__global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
                                                                         uint64_t count,
                                                                         const uint32_t* __restrict__ ids,
                                                                         uint32_t W, SampleCtl* ctl,
@@ -244,7 +262,7 @@ __global__ void __launch_bounds__(G == 512 ? 512 : 256) ic_group_kernel(GraphVie
     if (s_local == 0xFFFFFFFFu) break;
     unsigned long long se = 0;
     uint32_t size = 0;
-    const uint32_t flag = ic_group_sample<G>(g, K, R, s_local, tier, ring, W, rw, gc, gtid, gi, se, size);
+    const uint32_t flag = ic_group_sample<G, (G >= 512 ? 1 : IC_U)>(g, K, R, s_local, tier, ring, W, rw, gc, gtid, gi, se, size);
     if (gtid == 0) {
       if (flag == 0) {
         R.sizes[s_local] = size;
@@ -343,8 +361,6 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
   }
 }
 
-constexpr int IC_G = 128;          // threads per sample, tier 1
-constexpr int IC_NG = 2;           // groups per block
 constexpr uint32_t IC_W = 1024;    // shared-memory frontier ring per group
 constexpr int IC_G2 = 512;         // tier 2 (global ring of capacity >= n)
 
@@ -457,10 +473,16 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
       slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count);
       ctx->tier_queue.reserve(slots * (uint64_t)W2 * 4, false, st);
       EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
+      EIM_CUDA(cudaEventRecord(ctx->ev0, st));
       launch_ic<IC_G2, true>(ctx, g, seed, R, nretry, ctx->retry_a.as<uint32_t>(), W2, ctl, nullptr,
                              ctx->tier_queue.as<uint32_t>(), 1, slots);
+      EIM_CUDA(cudaEventRecord(ctx->ev1, st));
       EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
       EIM_CUDA(cudaStreamSynchronize(st));
+      float ms2 = 0;
+      EIM_CUDA(cudaEventElapsedTime(&ms2, ctx->ev0, ctx->ev1));
+      res.kernel_ms += ms2;
+      res.launches++;
       edges += h->edges;
       table_full = h->arena_fail != 0;
       if (!table_full && h->retry_count) fail(EIM_E_CUDA, "tier-2 sampler failed with a ring of capacity n");

@@ -1,35 +1,75 @@
 // select.cu -- greedy max-coverage NodeSelection (Alg. 3).
 //
-// Per pick j (two kernels, no host round trip):
-//   argmax_kernel: key(x) = C[x] << 32 | (2^32-1-x) maximised over the grid
-//     (block reduce + one 64-bit atomicMax per block): highest count, ties to
-//     the lowest id (R10).  Already-selected vertices are excluded: the
-//     previous pick by index, older picks because their count was replaced by
-//     a sentinel.
-//   cover_kernel: v = argmax; for every set i in v's inverted list with
-//     F[i] = 0: F[i] <- 1 and C[x] -= 1 for each member x (Alg. 3 l.7-12).
-// Instead of the paper's thread-per-set binary search over all theta sets
-// (P:186), the sets containing v are found through an inverted index
-// (vertex -> set ids) built once per NodeSelection by a counting sort on C,
-// so a pick touches only the sets that contain v.
+// Per NodeSelection (all of R, from scratch, R15):
+//   1. candidates = vertices with C[v] > 0, compacted in ascending id order
+//      (stable scan), so a candidate index orders like its vertex id;
+//   2. the arena is remapped to candidate indices and an inverted index
+//      (candidate -> ids of the sets containing it) is built by a counting
+//      sort, so a pick touches only the sets that contain it (instead of the
+//      paper's thread-per-set binary search over all theta sets);
+//   3. ONE cooperative persistent kernel runs all k picks.  Per pick: every
+//      block reduces its slice of the working counts W to a 64-bit key
+//      (count << 32 | ~index: highest count, ties to the lowest id, R10), a
+//      grid barrier, every block reduces the block maxima, the winner's
+//      uncovered sets are marked covered (F[i] <- 1) and every member count is
+//      decremented (Alg. 3 l.7-12) by one warp per inverted-list entry, a
+//      grid barrier.  A selected vertex ends with W = 0 (all its sets are
+//      covered); when the maximum count is 0 every set is covered and the
+//      pick is the lowest unselected vertex id (R10).
+#include <cooperative_groups.h>
+
 #include <cub/cub.cuh>
 
 #include "eim_internal.h"
+
+namespace cg = cooperative_groups;
 
 namespace eim {
 
 namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
+constexpr int GB = 256;  // threads per block of the greedy kernel
 
-__global__ void count_to_u64_kernel(const uint32_t* __restrict__ C, uint32_t n, uint64_t* __restrict__ out) {
+__global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t* __restrict__ flags) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= n; i += stride)
-    out[i] = i < n ? (uint64_t)C[i] : 0ull;
+    flags[i] = (i < n && C[i] > 0u) ? 1u : 0u;
 }
 
-// inverted index fill: one warp per set, inv[fill[x]++] = set id
-__global__ void invert_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,
+// pos = exclusive scan of flags: candidate index of v
+__global__ void compact_kernel(const uint32_t* __restrict__ C, const uint32_t* __restrict__ pos, uint32_t n,
+                               uint32_t nc_pad, uint32_t* __restrict__ cand, uint32_t* __restrict__ cidx,
+                               uint32_t* __restrict__ W) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint32_t nc = pos[n];
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+    const uint32_t c = C[v];
+    if (c > 0u) {
+      const uint32_t p = pos[v];
+      cand[p] = (uint32_t)v;
+      cidx[v] = p;
+      W[p] = c;
+    }
+  }
+  for (uint64_t i = nc + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nc_pad; i += stride) W[i] = 0u;
+}
+
+__global__ void remap_kernel(const uint32_t* __restrict__ arena, uint64_t total, const uint32_t* __restrict__ cidx,
+                             uint32_t* __restrict__ arena_c) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride)
+    arena_c[i] = cidx[arena[i]];
+}
+
+__global__ void count_to_u64_kernel(const uint32_t* __restrict__ W, uint32_t nc, uint64_t* __restrict__ out) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= nc; i += stride)
+    out[i] = i < nc ? (uint64_t)W[i] : 0ull;
+}
+
+// inverted index fill: one warp per set, inv[fill[x]++] = set id (x = candidate index)
+__global__ void invert_kernel(const uint32_t* __restrict__ arena_c, const uint64_t* __restrict__ set_start,
                               const uint32_t* __restrict__ set_len, uint64_t num_sets,
                               unsigned long long* __restrict__ fill, uint32_t* __restrict__ inv) {
   const int lane = threadIdx.x & 31;
@@ -39,82 +79,110 @@ __global__ void invert_kernel(const uint32_t* __restrict__ arena, const uint64_t
     const uint64_t st = set_start[i];
     const uint32_t L = set_len[i];
     for (uint32_t t = lane; t < L; t += 32) {
-      const unsigned long long p = atomicAdd(&fill[arena[st + t]], 1ull);
+      const unsigned long long p = atomicAdd(&fill[arena_c[st + t]], 1ull);
       inv[p] = (uint32_t)i;
     }
   }
-}
-
-__global__ void init_work_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t n_pad,
-                                 uint32_t* __restrict__ W) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride)
-    W[i] = i < n ? C[i] : SENTINEL;
-}
-
-__device__ __forceinline__ unsigned long long vkey(uint32_t c, uint32_t x, uint32_t excl) {
-  return (c == SENTINEL || x == excl) ? 0ull : (((unsigned long long)c << 32) | (unsigned long long)(0xFFFFFFFFu - x));
 }
 
 __device__ __forceinline__ unsigned long long umax64(unsigned long long a, unsigned long long b) {
   return a > b ? a : b;
 }
 
-template <int BLOCK>
-__global__ void __launch_bounds__(BLOCK) argmax_kernel(const uint4* __restrict__ W4, uint32_t n4,
-                                                       const uint32_t* __restrict__ seeds, uint32_t j,
-                                                       unsigned long long* __restrict__ best) {
-  const uint32_t excl = j > 0 ? seeds[j - 1] : SENTINEL;
-  unsigned long long k = 0;
-  const uint32_t stride = gridDim.x * BLOCK;
-  for (uint32_t i = blockIdx.x * BLOCK + threadIdx.x; i < n4; i += stride) {
-    const uint4 c = W4[i];
-    const uint32_t x = i * 4u;
-    k = umax64(k, vkey(c.x, x, excl));
-    k = umax64(k, vkey(c.y, x + 1, excl));
-    k = umax64(k, vkey(c.z, x + 2, excl));
-    k = umax64(k, vkey(c.w, x + 3, excl));
-  }
+__device__ __forceinline__ unsigned long long ckey(uint32_t c, uint32_t i) {
+  return c ? (((unsigned long long)c << 32) | (unsigned long long)(0xFFFFFFFFu - i)) : 0ull;
+}
+
+__device__ __forceinline__ unsigned long long block_max(unsigned long long k, unsigned long long* red) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) k = umax64(k, __shfl_xor_sync(FULL, k, o));
-  __shared__ unsigned long long red[BLOCK / 32];
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = k;
   __syncthreads();
   if (threadIdx.x < 32) {
-    k = threadIdx.x < BLOCK / 32 ? red[threadIdx.x] : 0ull;
+    k = threadIdx.x < GB / 32 ? red[threadIdx.x] : 0ull;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) k = umax64(k, __shfl_xor_sync(FULL, k, o));
-    if (threadIdx.x == 0 && k) atomicMax(&best[j], k);
+    if (threadIdx.x == 0) red[0] = k;
   }
+  __syncthreads();
+  k = red[0];
+  __syncthreads();
+  return k;
 }
 
-__global__ void cover_kernel(uint32_t j, const unsigned long long* __restrict__ best,
-                             uint32_t* __restrict__ seeds, unsigned long long* __restrict__ gains,
-                             uint32_t* __restrict__ W, const uint64_t* __restrict__ inv_off,
-                             const uint32_t* __restrict__ inv, uint8_t* __restrict__ F,
-                             const uint64_t* __restrict__ set_start, const uint32_t* __restrict__ set_len,
-                             const uint32_t* __restrict__ arena) {
-  const unsigned long long key = best[j];
-  const uint32_t v = 0xFFFFFFFFu - (uint32_t)key;
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    seeds[j] = v;
-    gains[j] = key >> 32;
-    if (j > 0) W[seeds[j - 1]] = SENTINEL;  // its sets are all covered: nobody else touches it
-  }
-  // one warp per entry of v's inverted list: the covered sets are
-  // decremented in parallel across the whole grid
+struct GreedyArgs {
+  uint32_t k, nc_pad;
+  uint32_t* W;                  // working counts per candidate (padded with 0)
+  const uint32_t* cand;         // candidate -> vertex (ascending)
+  const uint64_t* inv_off;      // nc+1
+  const uint32_t* inv;          // set ids
+  uint8_t* F;                   // covered flags per set
+  const uint64_t* set_start;
+  const uint32_t* set_len;
+  const uint32_t* arena_c;      // arena in candidate indices
+  unsigned long long* blockmax; // gridDim
+  uint8_t* selected;            // n flags (for the all-covered case)
+  uint32_t* zc;                 // cursor of the lowest possibly-unselected id
+  uint32_t* seeds;
+  unsigned long long* gains;
+};
+
+__global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ unsigned long long red[GB / 32];
+  const uint32_t nc4 = a.nc_pad / 4;
+  const uint4* W4 = reinterpret_cast<const uint4*>(a.W);
   const int lane = threadIdx.x & 31;
-  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  const uint64_t lo = inv_off[v], hi = inv_off[v + 1];
-  for (uint64_t p = lo + warp; p < hi; p += nwarps) {
-    const uint32_t i = inv[p];
-    if (F[i]) continue;  // covered by an earlier pick (set ids are unique within v's list)
-    __syncwarp();
-    if (lane == 0) F[i] = 1;
-    const uint64_t st = set_start[i];
-    const uint32_t L = set_len[i];
-    for (uint32_t t = lane; t < L; t += 32) atomicSub(&W[arena[st + t]], 1u);
+  const uint64_t warp = ((uint64_t)blockIdx.x * GB + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * GB) >> 5;
+  for (uint32_t j = 0; j < a.k; ++j) {
+    // ---- argmax over this block's slice
+    unsigned long long km = 0;
+    for (uint32_t i = blockIdx.x * GB + threadIdx.x; i < nc4; i += gridDim.x * GB) {
+      const uint4 c = W4[i];
+      const uint32_t x = 4u * i;
+      km = umax64(km, ckey(c.x, x));
+      km = umax64(km, ckey(c.y, x + 1));
+      km = umax64(km, ckey(c.z, x + 2));
+      km = umax64(km, ckey(c.w, x + 3));
+    }
+    km = block_max(km, red);
+    if (threadIdx.x == 0) a.blockmax[blockIdx.x] = km;
+    grid.sync();
+    km = 0;
+    for (uint32_t b = threadIdx.x; b < gridDim.x; b += GB) km = umax64(km, a.blockmax[b]);
+    km = block_max(km, red);
+    if (km == 0ull) {
+      // every set is covered: the lowest unselected vertex id, gain 0
+      if (blockIdx.x == 0 && threadIdx.x == 0) {
+        uint32_t z = *a.zc;
+        while (a.selected[z]) ++z;
+        *a.zc = z;
+        a.selected[z] = 1;
+        a.seeds[j] = z;
+        a.gains[j] = 0;
+      }
+    } else {
+      const uint32_t ci = 0xFFFFFFFFu - (uint32_t)km;
+      if (blockIdx.x == 0 && threadIdx.x == 0) {
+        const uint32_t v = a.cand[ci];
+        a.selected[v] = 1;
+        a.seeds[j] = v;
+        a.gains[j] = km >> 32;
+      }
+      // ---- cover: one warp per entry of the winner's inverted list
+      const uint64_t lo = a.inv_off[ci], hi = a.inv_off[ci + 1];
+      for (uint64_t p = lo + warp; p < hi; p += nwarps) {
+        const uint32_t i = a.inv[p];
+        if (a.F[i]) continue;  // covered by an earlier pick (ids are unique within one list)
+        __syncwarp();
+        if (lane == 0) a.F[i] = 1;
+        const uint64_t st = a.set_start[i];
+        const uint32_t L = a.set_len[i];
+        for (uint32_t t = lane; t < L; t += 32) atomicSub(&a.W[a.arena_c[st + t]], 1u);
+      }
+    }
+    grid.sync();
   }
 }
 
@@ -123,54 +191,82 @@ __global__ void cover_kernel(uint32_t j, const unsigned long long* __restrict__ 
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
                 uint64_t* gains_out) {
   cudaStream_t st = ctx->stream;
-  const uint32_t n_pad = (n + 3u) & ~3u;
-  // ---- inverted index: inv_off = exclusive scan of C_total, then scatter set ids
-  ctx->inv_off.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);
-  ctx->inv_fill.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);
-  uint64_t* inv_off = ctx->inv_off.as<uint64_t>();
-  count_to_u64_kernel<<<grid_for(ctx, (uint64_t)n + 1, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), n, inv_off);
+  uint64_t* h64 = static_cast<uint64_t*>(ctx->h_pinned);
+  const uint64_t total = arena_cursor(ctx);  // arena elements of sets [0, num_sets)
+  // ---- 1. candidates (C > 0) in ascending id order
+  ctx->inv_fill.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);  // scratch: flags/pos (u32)
+  uint32_t* pos = ctx->inv_fill.as<uint32_t>();
+  flag_kernel<<<grid_for(ctx, (uint64_t)n + 1, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), n, pos);
   EIM_CUDA(cudaGetLastError());
   size_t tmp = 0;
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, inv_off, inv_off, (uint64_t)n + 1, st));
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, pos, pos, (uint64_t)n + 1, st));
   ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, inv_off, inv_off, (uint64_t)n + 1, st));
-  EIM_CUDA(cudaMemcpyAsync(ctx->inv_fill.p, inv_off, ((uint64_t)n + 1) * sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
-  EIM_CUDA(cudaMemcpyAsync(ctx->h_pinned, inv_off + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, pos, pos, (uint64_t)n + 1, st));
+  uint32_t* h32 = reinterpret_cast<uint32_t*>(h64 + 8);
+  EIM_CUDA(cudaMemcpyAsync(h32, pos + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
-  const uint64_t total = *static_cast<uint64_t*>(ctx->h_pinned);
+  const uint32_t nc = *h32;
+  const uint32_t nc_pad = (nc + 3u) & ~3u;
+  ctx->cand.reserve((uint64_t)std::max(nc, 1u) * 4, false, st);
+  ctx->cidx.reserve((uint64_t)n * 4, false, st);
+  ctx->C_work.reserve((uint64_t)std::max(nc_pad, 4u) * 4, false, st);
+  compact_kernel<<<grid_for(ctx, n, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), pos, n, nc_pad,
+                                                          ctx->cand.as<uint32_t>(), ctx->cidx.as<uint32_t>(),
+                                                          ctx->C_work.as<uint32_t>());
+  EIM_CUDA(cudaGetLastError());
+  // ---- 2. arena in candidate indices + inverted index
+  ctx->arena_c.reserve(std::max<uint64_t>(total, 1) * 4, false, st);
+  if (total)
+    remap_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(ctx->arena.as<uint32_t>(), total, ctx->cidx.as<uint32_t>(),
+                                                              ctx->arena_c.as<uint32_t>());
+  ctx->inv_off.reserve(((uint64_t)nc + 1) * sizeof(uint64_t), false, st);
+  uint64_t* inv_off = ctx->inv_off.as<uint64_t>();
+  count_to_u64_kernel<<<grid_for(ctx, (uint64_t)nc + 1, 256), 256, 0, st>>>(ctx->C_work.as<uint32_t>(), nc, inv_off);
+  EIM_CUDA(cudaGetLastError());
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, inv_off, inv_off, (uint64_t)nc + 1, st));
+  ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, inv_off, inv_off, (uint64_t)nc + 1, st));
+  ctx->stage_c.reserve(((uint64_t)nc + 1) * sizeof(uint64_t), false, st);
+  EIM_CUDA(cudaMemcpyAsync(ctx->stage_c.p, inv_off, ((uint64_t)nc + 1) * sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
   ctx->inv.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
-  if (num_sets > 0) {
+  if (num_sets > 0 && total > 0) {
     invert_kernel<<<grid_for(ctx, num_sets * 32, 256), 256, 0, st>>>(
-        ctx->arena.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), num_sets,
-        ctx->inv_fill.as<unsigned long long>(), ctx->inv.as<uint32_t>());
+        ctx->arena_c.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), num_sets,
+        ctx->stage_c.as<unsigned long long>(), ctx->inv.as<uint32_t>());
     EIM_CUDA(cudaGetLastError());
   }
-  // ---- working counts, covered flags, per-pick argmax slots
-  ctx->C_work.reserve((uint64_t)n_pad * sizeof(uint32_t), false, st);
+  // ---- 3. the k picks in one cooperative kernel
   ctx->covered.reserve(std::max<uint64_t>(num_sets, 1), false, st);
-  ctx->best.reserve((uint64_t)k * sizeof(unsigned long long), false, st);
+  ctx->selected.reserve((uint64_t)n + 4, false, st);
   ctx->seeds.reserve((uint64_t)k * sizeof(uint32_t), false, st);
   ctx->gains.reserve((uint64_t)k * sizeof(unsigned long long), false, st);
-  uint32_t* W = ctx->C_work.as<uint32_t>();
-  init_work_kernel<<<grid_for(ctx, n_pad, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), n, n_pad, W);
-  EIM_CUDA(cudaGetLastError());
   EIM_CUDA(cudaMemsetAsync(ctx->covered.p, 0, std::max<uint64_t>(num_sets, 1), st));
-  EIM_CUDA(cudaMemsetAsync(ctx->best.p, 0, (uint64_t)k * sizeof(unsigned long long), st));
-  ctx->kernel_launches += 5;
-  const uint32_t n4 = n_pad / 4;
-  constexpr int AB = 256;
-  const uint32_t ablocks = grid_for(ctx, n4, AB, 8);
-  const uint32_t cblocks = (uint32_t)ctx->sm_count * 8;
-  for (uint32_t j = 0; j < k; ++j) {
-    argmax_kernel<AB><<<ablocks, AB, 0, st>>>(reinterpret_cast<const uint4*>(W), n4, ctx->seeds.as<uint32_t>(), j,
-                                              ctx->best.as<unsigned long long>());
-    cover_kernel<<<cblocks, 256, 0, st>>>(j, ctx->best.as<unsigned long long>(), ctx->seeds.as<uint32_t>(),
-                                          ctx->gains.as<unsigned long long>(), W, inv_off, ctx->inv.as<uint32_t>(),
-                                          ctx->covered.as<uint8_t>(), ctx->set_start.as<uint64_t>(),
-                                          ctx->set_len.as<uint32_t>(), ctx->arena.as<uint32_t>());
-  }
-  EIM_CUDA(cudaGetLastError());
-  ctx->kernel_launches += 2ull * k;
+  EIM_CUDA(cudaMemsetAsync(ctx->selected.p, 0, (uint64_t)n + 4, st));
+  int per_sm = 0;
+  EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
+  uint32_t blocks = (uint32_t)std::max(1, std::min(per_sm, 4)) * ctx->sm_count;
+  ctx->best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
+  uint32_t* zc = reinterpret_cast<uint32_t*>(ctx->best.as<unsigned long long>() + blocks);
+  EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
+  GreedyArgs a;
+  a.k = k;
+  a.nc_pad = nc_pad;
+  a.W = ctx->C_work.as<uint32_t>();
+  a.cand = ctx->cand.as<uint32_t>();
+  a.inv_off = inv_off;
+  a.inv = ctx->inv.as<uint32_t>();
+  a.F = ctx->covered.as<uint8_t>();
+  a.set_start = ctx->set_start.as<uint64_t>();
+  a.set_len = ctx->set_len.as<uint32_t>();
+  a.arena_c = ctx->arena_c.as<uint32_t>();
+  a.blockmax = ctx->best.as<unsigned long long>();
+  a.selected = ctx->selected.as<uint8_t>();
+  a.zc = zc;
+  a.seeds = ctx->seeds.as<uint32_t>();
+  a.gains = ctx->gains.as<unsigned long long>();
+  void* args[] = {&a};
+  EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
+  ctx->kernel_launches += 9;
   std::vector<unsigned long long> g(k);
   EIM_CUDA(cudaMemcpyAsync(seeds_out, ctx->seeds.p, (uint64_t)k * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaMemcpyAsync(g.data(), ctx->gains.p, (uint64_t)k * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
