@@ -280,6 +280,233 @@ __global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed,
   if ((threadIdx.x & 31) == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
 
+// ---------------------------------------------------------------- fused IC
+// Tier 1: one block traverses MANY samples at once (fused traversals).  The
+// block keeps up to FS active samples in shared-memory slots; its frontier
+// ring holds (slot, vertex) entries of all of them.  Each batch takes up to
+// FG entries from the ring -- whatever samples they belong to -- merges their
+// in-rows into one Philox-quad space and sweeps it with all FG threads, so
+// the batch stays full while light samples come and go, and a heavy sample
+// (a long chain of hub expansions) advances one frontier batch per iteration
+// without holding back the rest.  Before each batch, free slots are refilled
+// with new sample ids from the launch ticket (up to one per thread).
+constexpr int FG = 512;                 // threads per block
+constexpr int FS = 512;                 // sample slots per block
+constexpr uint32_t FW = 4096;           // frontier ring entries per block
+constexpr int FU = 2;                   // quads per thread per sweep iteration
+
+struct FusedSlot {
+  uint32_t s_local, members, pending, flag;
+  unsigned long long edges;
+};
+
+struct FusedShared {
+  FusedSlot slot[FS];
+  uint32_t ring_v[FW];
+  uint16_t ring_s[FW];
+  unsigned long long q0[FG];
+  uint32_t qend[FG], nq[FG], T[FG];
+  uint16_t rslot[FG];
+  uint8_t wlo[FG], whi[FG];
+  uint16_t free_stack[FS];
+  uint32_t free_count, tail, exhausted, wsum[FG / 32];
+  unsigned long long t0;
+};
+
+__global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
+                                                      SampleCtl* ctl, uint32_t* retry_out) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  FusedShared& S = *reinterpret_cast<FusedShared*>(smem_raw);
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const PhiloxKey K = philox_key(seed);
+  for (int i = tid; i < FS; i += FG) S.free_stack[i] = (uint16_t)(FS - 1 - i);
+  if (tid == 0) {
+    S.free_count = FS;
+    S.tail = 0;
+    S.exhausted = 0;
+  }
+  __syncthreads();
+  uint32_t head = 0;
+  unsigned long long edges_acc = 0;
+  for (;;) {
+    // ---- (1) refill free slots with new samples while the backlog is short
+    uint32_t tail = S.tail;
+    const uint32_t backlog = tail - head;
+    uint32_t want = 0;
+    if (!S.exhausted && backlog < (uint32_t)FG) want = min(S.free_count, (uint32_t)FG - backlog);
+    __syncthreads();  // everyone has read free_count / tail / exhausted
+    if (want > 0) {
+      if (tid == 0) {
+        const unsigned long long t0 = atomicAdd(&ctl->ticket, (unsigned long long)want);
+        S.t0 = t0;
+        if (t0 + want >= count) S.exhausted = 1;
+      }
+      __syncthreads();
+      const unsigned long long t0 = S.t0;
+      const uint32_t got = t0 >= count ? 0u : (uint32_t)min((unsigned long long)want, count - t0);
+      if ((uint32_t)tid < got) {
+        const uint16_t sl = S.free_stack[S.free_count - 1 - tid];
+        const uint32_t s_local = (uint32_t)(t0 + tid);
+        const uint32_t root = draw_root(R.base + s_local, g.n, K);
+        const int r = table_insert(R.keys, R.bits, table_key(s_local, 0, root));
+        FusedSlot& q = S.slot[sl];
+        q.s_local = s_local;
+        q.members = 1;
+        q.pending = 1;
+        q.flag = r < 0 ? FLAG_TABLE : 0u;
+        q.edges = 0;
+        S.ring_v[(tail + tid) & (FW - 1)] = root;
+        S.ring_s[(tail + tid) & (FW - 1)] = sl;
+      }
+      __syncthreads();
+      if (tid == 0) {
+        S.free_count -= got;
+        S.tail = tail + got;
+      }
+      __syncthreads();
+      tail = S.tail;
+    }
+    if (head == tail) {
+      if (S.exhausted) break;  // uniform: all threads read the same shared words after a barrier
+      continue;
+    }
+    // ---- (2) stage the rows of up to FG frontier entries
+    const uint32_t nb = min((uint32_t)FG, tail - head);
+    uint32_t nq = 0;
+    if ((uint32_t)tid < nb) {
+      const uint32_t e = (head + tid) & (FW - 1);
+      const uint32_t u = S.ring_v[e];
+      const uint16_t sl = S.ring_s[e];
+      S.rslot[tid] = sl;
+      if (S.slot[sl].flag == 0) {  // rows of failed samples are skipped
+        const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
+        if (e1 > e0) {
+          nq = (uint32_t)(((e1 - 1) >> 2) - (e0 >> 2) + 1);
+          S.q0[tid] = e0 >> 2;
+          S.wlo[tid] = (uint8_t)(e0 & 3);
+          S.whi[tid] = (uint8_t)((e1 - 1) & 3);
+          S.T[tid] = g.thr[u];
+        }
+        atomicAdd(&S.slot[sl].edges, e1 - e0);
+      }
+      S.nq[tid] = nq;
+    }
+    // block inclusive scan of nq
+    uint32_t x = nq;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += t;
+    }
+    if (lane == 31) S.wsum[wid] = x;
+    __syncthreads();
+    uint32_t pre = 0, total = 0;
+#pragma unroll
+    for (int i = 0; i < FG / 32; ++i) {
+      const uint32_t t = S.wsum[i];
+      pre += (i < wid) ? t : 0u;
+      total += t;
+    }
+    if ((uint32_t)tid < nb) S.qend[tid] = x + pre;
+    head += nb;
+    __syncthreads();
+    // ---- (3) sweep the merged quad space
+    int r = -1;
+    uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0, sl_r = 0, sloc_r = 0;
+    unsigned long long q0_r = 0;
+    for (uint32_t base = 0; base < total; base += FU * FG) {
+      unsigned long long qk[FU];
+      uint32_t Tk[FU], mk[FU], slk[FU], sk[FU];
+#pragma unroll
+      for (int k = 0; k < FU; ++k) {
+        const uint32_t j = base + k * FG + tid;
+        mk[k] = 0u;
+        qk[k] = 0ull;
+        Tk[k] = 0u;
+        slk[k] = 0u;
+        sk[k] = 0u;
+        if (j < total) {
+          if (j >= qe) {
+            do {
+              ++r;
+              qe = S.qend[r];
+            } while (j >= qe);
+            nq_r = S.nq[r];
+            qb = qe - nq_r;
+            q0_r = S.q0[r];
+            T_r = S.T[r];
+            wlo_r = S.wlo[r];
+            whi_r = S.whi[r];
+            sl_r = S.rslot[r];
+            sloc_r = S.slot[sl_r].s_local;
+          }
+          const uint32_t li = j - qb;
+          uint32_t m = 0xFu;
+          if (li == 0) m &= 0xFu << wlo_r;
+          if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
+          mk[k] = m;
+          qk[k] = q0_r + li;
+          Tk[k] = T_r;
+          slk[k] = sl_r;
+          sk[k] = sloc_r;
+        }
+      }
+      uint4 wk[FU];
+#pragma unroll
+      for (int k = 0; k < FU; ++k) wk[k] = philox_at(qk[k], R.base + sk[k], TAG_EDGE, K);
+#pragma unroll
+      for (int k = 0; k < FU; ++k) {
+        const uint32_t T = Tk[k];
+        uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
+                        (wk[k].w <= T ? 8u : 0u);
+        live &= mk[k];
+        while (live) {
+          const int i = __ffs(live) - 1;
+          live &= live - 1;
+          const uint32_t v = g.nbr[(qk[k] << 2) + i];
+          FusedSlot& q = S.slot[slk[k]];
+          const int ins = table_insert(R.keys, R.bits, table_key(sk[k], 0, v));
+          if (ins > 0) {
+            atomicAdd(&q.members, 1u);
+            const uint32_t pos = atomicAdd(&S.tail, 1u);
+            if (pos - head < FW) {
+              atomicAdd(&q.pending, 1u);
+              S.ring_v[pos & (FW - 1)] = v;
+              S.ring_s[pos & (FW - 1)] = (uint16_t)slk[k];
+            } else {
+              atomicOr(&q.flag, FLAG_RING);  // entry lost: the sample is redone by tier 2
+            }
+          } else if (ins < 0) {
+            atomicOr(&q.flag, FLAG_TABLE);
+          }
+        }
+      }
+    }
+    __syncthreads();
+    // ---- (4) retire the batch's entries; a sample with nothing pending is done
+    if ((uint32_t)tid < nb) {
+      const uint16_t sl = S.rslot[tid];
+      FusedSlot& q = S.slot[sl];
+      if (atomicSub(&q.pending, 1u) == 1u) {
+        const uint32_t f = q.flag;
+        if (f == 0u) {
+          R.sizes[q.s_local] = q.members;
+          edges_acc += q.edges;
+        } else if (f & FLAG_TABLE) {
+          atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);
+        } else {
+          R.failed[q.s_local] = 1;
+          retry_out[atomicAdd(&ctl->retry_count, 1ull)] = q.s_local;
+        }
+        S.free_stack[atomicAdd(&S.free_count, 1u)] = sl;
+      }
+    }
+    __syncthreads();
+  }
+  for (int o = 16; o > 0; o >>= 1) edges_acc += __shfl_xor_sync(FULL, edges_acc, o);
+  if (lane == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
+}
+
 // ---------------------------------------------------------------- LT
 // Reverse LT walk (R3-R5): at u with d^-(u) > 0, tau_u is the
 // LT-tagged draw of u and the chosen in-neighbour is position
@@ -444,8 +671,16 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
     EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
     EIM_CUDA(cudaEventRecord(ctx->ev0, st));
     if (model == EIM_IC) {
-      launch_ic<IC_G, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr,
-                             IC_NG, ~0ull);
+      const size_t smem = sizeof(FusedShared);
+      EIM_CUDA(cudaFuncSetAttribute(ic_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      int per_sm = 0;
+      EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ic_fused_kernel, FG, smem));
+      uint64_t blocks = (uint64_t)std::max(1, per_sm) * ctx->sm_count;
+      blocks = std::min<uint64_t>(blocks, (count + 63) / 64);
+      ic_fused_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), FG, smem, st>>>(g->view, seed, R, count, ctl,
+                                                                                   ctx->retry_a.as<uint32_t>());
+      EIM_CUDA(cudaGetLastError());
+      ctx->kernel_launches++;
     } else {
       int per_sm = 0;
       EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel, 256, 0));
