@@ -158,6 +158,12 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
                             const uint32_t* members, uint32_t k, uint32_t* seeds_out,
                             uint64_t* gains_out);
 
+/* Statistics of the most recent eim_imm_run / eim_sample_rrr call on ctx
+ * (for eim_sample_rrr: theta = count, edges_examined, sample_launches,
+ * tier2_samples, ms_sample_kernel, ms_sample, ms_total, arena_elems,
+ * kernel_launches).  Errors: EIM_E_STATE, EIM_E_INVAL (out NULL). */
+eim_status eim_get_stats(const eim_ctx* ctx, eim_stats* out);
+
 /* ---------------------------------------------------------------- host-only
  * These need no device and may be called with no context. */
 /* IMM parameters (formulas above; R17 fixes the evaluation order).

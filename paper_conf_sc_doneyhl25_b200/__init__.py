@@ -27,7 +27,7 @@ STATUS_NAMES = {0: "EIM_OK", -1: "EIM_E_INVAL", -2: "EIM_E_NOMEM", -3: "EIM_E_CU
 # Every symbol include/eim.h declares (checked by tests/test_abi.py).
 EXPORTS = ["eim_create", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "eim_version",
            "eim_load_graph_csr", "eim_graph_free", "eim_imm_run", "eim_sample_rrr", "eim_select_seeds",
-           "eim_imm_params", "eim_shard_range"]
+           "eim_imm_params", "eim_shard_range", "eim_get_stats"]
 
 
 class EimError(RuntimeError):
@@ -96,6 +96,7 @@ def lib():
         "eim_select_seeds": (_I, [_P, _U32, _U64, _P, _P, _U32, _P, _P]),
         "eim_imm_params": (_I, [_U32, _U32, _D, _D, ctypes.POINTER(ImmParams)]),
         "eim_shard_range": (_I, [_U64, _U64, _I, _I, ctypes.POINTER(_U64), ctypes.POINTER(_U64)]),
+        "eim_get_stats": (_I, [_P, _P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -202,6 +203,12 @@ def eim_select_seeds(ctx, n, offsets, members, k):
     _check(lib().eim_select_seeds(ctx, n, off.size - 1, off.ctypes.data, mem.ctypes.data if mem.size else None, k,
                                   seeds.ctypes.data, gains.ctypes.data), ctx)
     return seeds, gains
+
+
+def eim_get_stats(ctx):
+    st = Stats()
+    _check(lib().eim_get_stats(ctx, ctypes.addressof(st)), ctx)
+    return st.as_dict()
 
 
 # ------------------------------------------------------------------ host-only

@@ -92,7 +92,7 @@ void free_ctx_buffers(eim_ctx* c) {
                     &c->tier_tab, &c->tier_queue, &c->tier_gen, &c->C_total, &c->C_work, &c->inv_off,
                     &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
                     &c->stage_b, &c->stage_c, &c->table, &c->rsizes, &c->rfailed, &c->rfill,
-                    &c->cand, &c->cidx, &c->arena_c, &c->selected};
+                    &c->cand, &c->cidx, &c->arena_c, &c->selected, &c->pool, &c->pool_ctl};
   for (DevBuf* b : bufs) b->release();
 }
 
@@ -238,8 +238,8 @@ eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps,
     if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
     if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
-    eim_stats local;
-    imm_run(ctx, g, k, eps, ell, model, seed, seeds_out, theta_out, spread_out, stats_out ? stats_out : &local);
+    imm_run(ctx, g, k, eps, ell, model, seed, seeds_out, theta_out, spread_out, &ctx->last_stats);
+    if (stats_out) *stats_out = ctx->last_stats;
   });
 }
 
@@ -254,8 +254,17 @@ eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
     if (first_id + count < first_id || first_id + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids must be < 2^62");
     cudaStream_t st = ctx->stream;
+    const auto t0 = std::chrono::steady_clock::now();
+    const uint64_t launches0 = ctx->kernel_launches;
     arena_reset(ctx);
-    sample_range(ctx, g, model, seed, first_id, count, first_id, false);
+    const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false);
+    std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
+    ctx->last_stats.edges_examined = r.edges;
+    ctx->last_stats.tier2_samples = r.tier2;
+    ctx->last_stats.sample_launches = r.launches;
+    ctx->last_stats.ms_sample_kernel = r.kernel_ms;
+    ctx->last_stats.theta = count;
+    ctx->last_stats.ms_sample = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     uint64_t* d_off = nullptr;
     uint32_t* d_mem = nullptr;
     const uint64_t total = export_sets(ctx, count, &d_off, &d_mem);
@@ -272,6 +281,9 @@ eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
       EIM_CUDA(cudaMemcpyAsync(members_out, d_mem, total * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
     }
     EIM_CUDA(cudaStreamSynchronize(st));
+    ctx->last_stats.arena_elems = total;
+    ctx->last_stats.kernel_launches = ctx->kernel_launches - launches0;
+    ctx->last_stats.ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   });
   return s != EIM_OK ? s : cap_status;
 }
@@ -302,6 +314,13 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     hist_sets(ctx, 0, num_sets);
     greedy(ctx, n, num_sets, k, seeds_out, gains_out);
   });
+}
+
+eim_status eim_get_stats(const eim_ctx* ctx, eim_stats* out) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  if (!out) return EIM_E_INVAL;
+  *out = ctx->last_stats;
+  return EIM_OK;
 }
 
 eim_status eim_imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out) {

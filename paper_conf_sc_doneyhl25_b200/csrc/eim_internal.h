@@ -89,6 +89,9 @@ struct eim_ctx {
   eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
   eim::DevBuf table, rsizes, rfailed, rfill;    // per-round membership table + per-sample scratch
   double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
+  eim::DevBuf pool, pool_ctl;                   // IC task pool (chunk tasks) + its counters
+  double est_chunks_per_sample = 0;
+  uint64_t pool_dirty = 0, pool_cap_hint = 0;
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;
@@ -97,6 +100,7 @@ struct eim_ctx {
   eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
   void* h_pinned = nullptr;   // small pinned host scratch
   cudaEvent_t ev0, ev1;
+  eim_stats last_stats;       // statistics of the most recent hot-path call
 };
 
 namespace eim {

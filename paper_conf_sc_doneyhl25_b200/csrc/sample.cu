@@ -25,6 +25,9 @@
 //   visited set = the same global table; no capacity limit.
 #include <cub/cub.cuh>
 
+#include <cstdlib>
+#include <string>
+
 #include "eim_internal.h"
 #include "philox.cuh"
 
@@ -314,7 +317,7 @@ struct FusedShared {
 };
 
 __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
-                                                      SampleCtl* ctl, uint32_t* retry_out) {
+                                                      SampleCtl* ctl, uint32_t* retry_out, uint32_t chunk) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   FusedShared& S = *reinterpret_cast<FusedShared*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -333,7 +336,7 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
     uint32_t tail = S.tail;
     const uint32_t backlog = tail - head;
     uint32_t want = 0;
-    if (!S.exhausted && backlog < (uint32_t)FG) want = min(S.free_count, (uint32_t)FG - backlog);
+    if (!S.exhausted && backlog < (uint32_t)FG) want = min(min(S.free_count, (uint32_t)FG - backlog), chunk);
     __syncthreads();  // everyone has read free_count / tail / exhausted
     if (want > 0) {
       if (tid == 0) {
@@ -507,6 +510,200 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
   if (lane == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
 
+// ---------------------------------------------------------------- pool IC
+// Tier 1 default: ONE global task pool per round, no per-sample on-chip
+// state.  A task is a chunk of at most PQ Philox quads of one in-row of one
+// sample: (s_local, first quad, quad count, edge-word masks, T).  Whoever
+// discovers a new member v of sample s (table insert succeeded) loads v's row
+// bounds and publishes ceil(quads / PQ) chunk tasks; any warp claims tasks,
+// merges the quads of its claimed tasks into one space swept by its 32 lanes,
+// and publishes the tasks of the members it discovers.  BFS order is
+// irrelevant to the result (the set is the reverse reachability of the root
+// in the live-edge world), so there are no levels and no barriers: a hub row
+// found in a deep chain is split across the whole GPU the moment it is found,
+// and the round ends when the count of unfinished tasks reaches zero.
+constexpr uint32_t PQ = 64;  // quads per chunk task
+
+struct PoolView {
+  ulonglong2* q;                 // task slots (zeroed; y != 0 marks a published task)
+  unsigned long long cap;
+  unsigned long long* head;      // claim counter
+  unsigned long long* tail;      // reservation counter
+  unsigned long long* pending;   // seeds not yet processed + tasks published and not yet finished
+  unsigned int* flags;           // bit 0: queue full, bit 1: table full, bit 2: watchdog
+};
+
+__device__ __forceinline__ void pool_push_row(const GraphView& g, const PoolView& P, uint32_t s_local, uint32_t v) {
+  const unsigned long long e0 = g.off[v], e1 = g.off[v + 1];
+  if (e1 == e0) return;
+  const unsigned long long q0 = e0 >> 2;
+  const unsigned long long nq = ((e1 - 1) >> 2) - q0 + 1;
+  const uint32_t T = g.thr[v];
+  const unsigned long long nch = (nq + PQ - 1) / PQ;
+  atomicAdd(P.pending, nch);
+  const unsigned long long base = atomicAdd(P.tail, nch);
+  unsigned long long ok = nch;
+  if (base + nch > P.cap) {
+    ok = base >= P.cap ? 0ull : P.cap - base;
+    atomicAdd(P.pending, 0ull - (nch - ok));
+    atomicOr(P.flags, 1u);
+  }
+  for (unsigned long long c = 0; c < ok; ++c) {
+    const unsigned long long cq0 = q0 + c * PQ;
+    P.q[base + c].x = (cq0 & 0xFFFFFFFFull) | ((unsigned long long)T << 32);
+  }
+  __threadfence();
+  for (unsigned long long c = 0; c < ok; ++c) {
+    const unsigned long long cq0 = q0 + c * PQ;
+    const uint32_t cn = (uint32_t)min((unsigned long long)PQ, nq - c * PQ);
+    const uint32_t wlo = c == 0 ? (uint32_t)(e0 & 3) : 0u;
+    const uint32_t whi = c == nch - 1 ? (uint32_t)((e1 - 1) & 3) : 3u;
+    const uint32_t meta = cn | (wlo << 16) | (whi << 18) | ((uint32_t)(cq0 >> 32) << 20);
+    *(volatile unsigned long long*)&P.q[base + c].y = (unsigned long long)meta | ((unsigned long long)(s_local + 1) << 32);
+  }
+}
+
+__global__ void __launch_bounds__(256) ic_pool_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
+                                                      PoolView P, SampleCtl* ctl, uint32_t total_warps) {
+  const int lane = threadIdx.x & 31;
+  const PhiloxKey K = philox_key(seed);
+  unsigned long long edges_acc = 0;
+  // ---- seeds: roots of the round's samples (Alg. 2 l.6-9)
+  for (;;) {
+    unsigned long long t0 = 0;
+    if (lane == 0) t0 = atomicAdd(&ctl->ticket, 32ull);
+    t0 = __shfl_sync(FULL, t0, 0);
+    if (t0 >= count) break;
+    const unsigned long long t = t0 + lane;
+    if (t < count) {
+      const uint32_t s_local = (uint32_t)t;
+      const uint32_t root = draw_root(R.base + s_local, g.n, K);
+      const int r = table_insert(R.keys, R.bits, table_key(s_local, 0, root));
+      if (r < 0) atomicOr(P.flags, 2u);
+      atomicAdd(&R.sizes[s_local], 1u);
+      pool_push_row(g, P, s_local, root);
+    }
+    const uint32_t nseed = (uint32_t)min(32ull, count - t0);
+    __threadfence();
+    __syncwarp();
+    if (lane == 0) atomicAdd(P.pending, 0ull - (unsigned long long)nseed);
+  }
+  // ---- tasks
+  unsigned long long spins = 0;
+  for (;;) {
+    // claim n consecutive slots; n adapts to the backlog so that in a thin
+    // tail consecutive tasks (the chunks of one hub row) go to different warps
+    unsigned long long h = 0, n = 0;
+    if (lane == 0) {
+      const unsigned long long hv = *(volatile unsigned long long*)P.head;
+      const unsigned long long tv = *(volatile unsigned long long*)P.tail;
+      const unsigned long long avail = tv > hv ? tv - hv : 0ull;
+      n = min(32ull, max(1ull, avail / total_warps));
+      h = atomicAdd(P.head, n);
+    }
+    h = __shfl_sync(FULL, h, 0);
+    n = __shfl_sync(FULL, n, 0);
+    bool mine = (unsigned long long)lane < n && h + lane < P.cap;
+    bool done = !mine;
+    for (;;) {
+      // wait until some claimed slot is published, or the round is over
+      unsigned long long y = 0;
+      if (!done) y = *(volatile unsigned long long*)&P.q[h + lane].y;
+      const bool ready = !done && y != 0ull;
+      const unsigned rmask = __ballot_sync(FULL, ready);
+      if (rmask == 0u) {
+        if (__ballot_sync(FULL, !done) == 0u) break;  // all claimed slots handled
+        unsigned long long pend = 0;
+        if (lane == 0) pend = *(volatile unsigned long long*)P.pending;
+        pend = __shfl_sync(FULL, pend, 0);
+        if (pend == 0ull) break;  // nothing will be published any more
+        if (++spins > (1ull << 26)) {
+          if (lane == 0) atomicOr(P.flags, 4u);
+          break;
+        }
+        __nanosleep(200);
+        continue;
+      }
+      __threadfence();
+      // decode this lane's task
+      uint32_t cn = 0, T = 0, wlo = 0, whi = 3, s_local = 0;
+      unsigned long long cq0 = 0;
+      if (ready) {
+        const unsigned long long x = __ldcg(&P.q[h + lane].x);
+        const uint32_t meta = (uint32_t)y;
+        s_local = (uint32_t)(y >> 32) - 1u;
+        cn = meta & 0xFFFFu;
+        wlo = (meta >> 16) & 3u;
+        whi = (meta >> 18) & 3u;
+        cq0 = (x & 0xFFFFFFFFull) | ((unsigned long long)(meta >> 20) << 32);
+        T = (uint32_t)(x >> 32);
+        edges_acc += 4ull * cn - wlo - (3u - whi);
+        done = true;
+      }
+      // merge the ready tasks' quads into one space swept by the warp
+      uint32_t incl = cn;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t v = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      const uint32_t total = __shfl_sync(FULL, incl, 31);
+      for (uint32_t base = 0; base < total; base += 32u) {
+        const uint32_t j = base + lane;
+        // owner lane of quad j: the first lane whose inclusive quad sum exceeds j
+        int src = 0;
+#pragma unroll
+        for (int b = 16; b > 0; b >>= 1) {
+          const uint32_t ib = __shfl_sync(FULL, incl, src + b - 1);
+          if (ib <= j) src += b;
+        }
+        const uint32_t r_incl = __shfl_sync(FULL, incl, src);
+        const uint32_t r_cn = __shfl_sync(FULL, cn, src);
+        const uint32_t r_T = __shfl_sync(FULL, T, src);
+        const uint32_t r_wlo = __shfl_sync(FULL, wlo, src);
+        const uint32_t r_whi = __shfl_sync(FULL, whi, src);
+        const uint32_t r_s = __shfl_sync(FULL, s_local, src);
+        const unsigned long long r_q0 = __shfl_sync(FULL, cq0, src);
+        if (j < total) {
+          const uint32_t li = j - (r_incl - r_cn);
+          const unsigned long long q = r_q0 + li;
+          const uint4 w = philox_at(q, R.base + r_s, TAG_EDGE, K);
+          uint32_t m = 0xFu;
+          if (li == 0) m &= 0xFu << r_wlo;
+          if (li == r_cn - 1) m &= 0xFu >> (3u - r_whi);
+          uint32_t live = (w.x <= r_T ? 1u : 0u) | (w.y <= r_T ? 2u : 0u) | (w.z <= r_T ? 4u : 0u) |
+                          (w.w <= r_T ? 8u : 0u);
+          live &= m;
+          while (live) {
+            const int i = __ffs(live) - 1;
+            live &= live - 1;
+            const uint32_t v = g.nbr[(q << 2) + i];
+            const int ins = table_insert(R.keys, R.bits, table_key(r_s, 0, v));
+            if (ins > 0) {
+              atomicAdd(&R.sizes[r_s], 1u);
+              pool_push_row(g, P, r_s, v);
+            } else if (ins < 0) {
+              atomicOr(P.flags, 2u);
+            }
+          }
+        }
+      }
+      // finished tasks leave the pending count only after their children
+      // were counted in (fence + warp barrier order the lanes' increments first)
+      __threadfence();
+      __syncwarp();
+      if (lane == 0) atomicAdd(P.pending, 0ull - (unsigned long long)__popc(rmask));
+    }
+    if (*(volatile unsigned int*)P.flags & 4u) break;
+    unsigned long long pend = 0;
+    if (lane == 0) pend = *(volatile unsigned long long*)P.pending;
+    pend = __shfl_sync(FULL, pend, 0);
+    if (pend == 0ull) break;
+  }
+  for (int o = 16; o > 0; o >>= 1) edges_acc += __shfl_xor_sync(FULL, edges_acc, o);
+  if (lane == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
+}
+
 // ---------------------------------------------------------------- LT
 // Reverse LT walk (R3-R5): at u with d^-(u) > 0, tau_u is the
 // LT-tagged draw of u and the chosen in-neighbour is position
@@ -668,17 +865,65 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
                 first};
     EIM_CUDA(cudaMemsetAsync(R.keys, 0, 8ull << bits, st));
     EIM_CUDA(cudaMemsetAsync(R.failed, 0, count, st));
+    EIM_CUDA(cudaMemsetAsync(R.sizes, 0, count * sizeof(uint32_t), st));
     EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
     EIM_CUDA(cudaEventRecord(ctx->ev0, st));
-    if (model == EIM_IC) {
+    const char* var = getenv("EIM_IC_KERNEL");  // development switch: "group" / "fused" / default "pool"
+    const std::string variant = var ? std::string(var) : std::string("pool");
+    if (model == EIM_IC && variant == "pool") {
+      // task pool capacity from the chunks per sample of earlier rounds
+      const double cps = ctx->est_chunks_per_sample > 0 ? ctx->est_chunks_per_sample : 256.0;
+      uint64_t cap = std::max<uint64_t>(1ull << 20, (uint64_t)(2.0 * cps * (double)count) + 4096);
+      if (attempt > 0) cap = std::max<uint64_t>(cap, ctx->pool_cap_hint);
+      const size_t old_bytes = ctx->pool.bytes;
+      ctx->pool.reserve(cap * 16, false, st);
+      cap = ctx->pool.bytes / 16;
+      if (ctx->pool.bytes != old_bytes) ctx->pool_dirty = cap;  // fresh allocation: zero all of it
+      const uint64_t dirty = std::min<uint64_t>(ctx->pool_dirty, cap);
+      if (dirty) EIM_CUDA(cudaMemsetAsync(ctx->pool.p, 0, dirty * 16, st));
+      ctx->pool_ctl.reserve(64, false, st);
+      unsigned long long* pc = ctx->pool_ctl.as<unsigned long long>();
+      unsigned long long* hpc = reinterpret_cast<unsigned long long*>(static_cast<char*>(ctx->h_pinned) + 2048);
+      hpc[0] = 0; hpc[1] = 0; hpc[2] = count; hpc[3] = 0;
+      EIM_CUDA(cudaMemcpyAsync(pc, hpc, 32, cudaMemcpyHostToDevice, st));
+      PoolView P{ctx->pool.as<ulonglong2>(), cap, pc, pc + 1, pc + 2, reinterpret_cast<unsigned int*>(pc + 3)};
+      int per_sm = 0;
+      EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ic_pool_kernel, 256, 0));
+      const uint32_t blocks = (uint32_t)std::max(1, per_sm) * ctx->sm_count;
+      ic_pool_kernel<<<blocks, 256, 0, st>>>(g->view, seed, R, count, P, ctl, blocks * 8);
+      EIM_CUDA(cudaGetLastError());
+      ctx->kernel_launches++;
+      EIM_CUDA(cudaMemcpyAsync(hpc, pc, 32, cudaMemcpyDeviceToHost, st));
+      EIM_CUDA(cudaStreamSynchronize(st));
+      const uint64_t used = hpc[1];
+      const unsigned int pflags = (unsigned int)hpc[3];
+      ctx->pool_dirty = std::max<uint64_t>(ctx->pool_dirty, std::min<uint64_t>(used, cap));
+      if (pflags & 4u) fail(EIM_E_CUDA, "sampler watchdog fired (task pool stalled)");
+      if (pflags & 1u) {  // task pool overflow: redo the round with a larger pool
+        ctx->pool_cap_hint = std::max<uint64_t>(cap * 2, used + used / 4);
+        if (attempt >= 6) fail(EIM_E_NOMEM, "task pool overflow");
+        continue;
+      }
+      if (pflags & 2u) {
+        if (attempt >= 4 || bits >= 31) fail(EIM_E_NOMEM, "membership table overflow");
+        bits += 2;
+        continue;
+      }
+      ctx->est_chunks_per_sample = std::max(1.0, (double)used / (double)count);
+    } else if (model == EIM_IC && variant == "group") {
+      launch_ic<IC_G, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr,
+                             IC_NG, ~0ull);
+    } else if (model == EIM_IC) {
       const size_t smem = sizeof(FusedShared);
       EIM_CUDA(cudaFuncSetAttribute(ic_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       int per_sm = 0;
       EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ic_fused_kernel, FG, smem));
       uint64_t blocks = (uint64_t)std::max(1, per_sm) * ctx->sm_count;
-      blocks = std::min<uint64_t>(blocks, (count + 63) / 64);
-      ic_fused_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), FG, smem, st>>>(g->view, seed, R, count, ctl,
-                                                                                   ctx->retry_a.as<uint32_t>());
+      blocks = std::max<uint64_t>(1, std::min<uint64_t>(blocks, count));
+      // new samples per block per batch: small enough that every block gets a share of the round
+      const uint32_t chunk = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(64, count / (blocks * 8)));
+      ic_fused_kernel<<<(uint32_t)blocks, FG, smem, st>>>(g->view, seed, R, count, ctl, ctx->retry_a.as<uint32_t>(),
+                                                          chunk);
       EIM_CUDA(cudaGetLastError());
       ctx->kernel_launches++;
     } else {
