@@ -25,6 +25,7 @@
 //   visited set = the same global table; no capacity limit.
 #include <cub/cub.cuh>
 
+#include <cstdio>
 #include <cstdlib>
 #include <string>
 
@@ -37,9 +38,16 @@ namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr uint32_t MAX_PROBE = 256;
+__device__ unsigned long long* g_dbg_group = nullptr;  // EIM_DEBUG_TIMES (development)
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 constexpr int IC_G = 256;          // threads per sample (one block), tier 1
 constexpr int IC_NG = 1;           // groups per block
-constexpr int IC_U = 2;            // quads per thread per sweep iteration
+constexpr int IC_U = 2;            // consecutive quads per thread per sweep iteration
 
 // ---------------------------------------------------------------- table
 // key = ((s_local + 1) | tier << 31) << 32 | v ;  0 = empty slot.
@@ -76,7 +84,7 @@ __device__ __forceinline__ void gsync(int) {
 
 struct GroupCtl {
   uint32_t tail, flag, s_local, pad;
-  uint32_t wsum[16];
+  uint32_t wsum[32];  // one per warp (G <= 1024)
 };
 
 template <int G>
@@ -143,13 +151,25 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
   gsync<G>(gi);
   uint32_t head = 0;
   se = 0;
+#ifdef EIM_DEV_TIMING
+  unsigned long long* dbg = g_dbg_group;
+#else
+  constexpr unsigned long long* dbg = nullptr;  // per-phase timing only in development builds
+#endif
+  unsigned long long t_begin = 0, t_stage = 0, t_sweep = 0, nbatch = 0, nquads = 0, ta = 0;
+  if (dbg && gtid == 0) t_begin = gtimer();
   for (;;) {
     const uint32_t tail = *(volatile uint32_t*)&gc.tail;
     const uint32_t flag = *(volatile uint32_t*)&gc.flag;
     if (flag || head >= tail) {
       size = tail;
+      if (dbg && gtid == 0 && tier == 0) {
+        unsigned long long* d = dbg + 6ull * s_local;
+        d[0] = t_begin; d[1] = gtimer(); d[2] = nbatch; d[3] = t_stage; d[4] = t_sweep; d[5] = nquads;
+      }
       return flag;
     }
+    if (dbg && gtid == 0) ta = gtimer();
     const uint32_t nb = min((uint32_t)G, tail - head);
     uint32_t nq = 0;
     if (gtid < nb) {
@@ -170,6 +190,8 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
     if (gtid < nb) rw.qend[gtid] = incl;
     head += nb;  // ring slots [old head, head) are free again: their rows are staged
     gsync<G>(gi);
+    unsigned long long tb = 0;
+    if (dbg && gtid == 0) { tb = gtimer(); t_stage += tb - ta; nbatch++; nquads += total; }
     // Sweep the batch's quad space; each thread takes U quads per iteration
     // (j, j+G, .., j+(U-1)G) whose Philox chains are independent (ILP).
     int r = -1;
@@ -231,6 +253,7 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
       }
     }
     gsync<G>(gi);
+    if (dbg && gtid == 0) t_sweep += gtimer() - tb;
   }
 }
 
@@ -265,7 +288,7 @@ __global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed,
     if (s_local == 0xFFFFFFFFu) break;
     unsigned long long se = 0;
     uint32_t size = 0;
-    const uint32_t flag = ic_group_sample<G, (G >= 512 ? 1 : IC_U)>(g, K, R, s_local, tier, ring, W, rw, gc, gtid, gi, se, size);
+    const uint32_t flag = ic_group_sample<G, IC_U>(g, K, R, s_local, tier, ring, W, rw, gc, gtid, gi, se, size);
     if (gtid == 0) {
       if (flag == 0) {
         R.sizes[s_local] = size;
@@ -296,11 +319,13 @@ __global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed,
 constexpr int FG = 512;                 // threads per block
 constexpr int FS = 512;                 // sample slots per block
 constexpr uint32_t FW = 4096;           // frontier ring entries per block
-constexpr int FU = 2;                   // quads per thread per sweep iteration
+constexpr int FU = 4;                   // consecutive quads per thread per sweep iteration
 
 struct FusedSlot {
   uint32_t s_local, members, pending, flag;
   unsigned long long edges;
+  unsigned long long t_start;  // debug timing (EIM_DEBUG_TIMES)
+  uint32_t levels, last_batch;
 };
 
 struct FusedShared {
@@ -316,8 +341,30 @@ struct FusedShared {
   unsigned long long t0;
 };
 
-__global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
-                                                      SampleCtl* ctl, uint32_t* retry_out, uint32_t chunk) {
+// A live in-edge reached v for the sample in slot sl: insert (sample, v) into
+// the round table; a new member joins the block's frontier ring.
+__device__ __forceinline__ void fused_visit(const GraphView& g, const RoundView& R, FusedShared& S, uint32_t v,
+                                            uint32_t sl, uint32_t sloc, uint32_t head) {
+  FusedSlot& q = S.slot[sl];
+  const int ins = table_insert(R.keys, R.bits, table_key(sloc, 0, v));
+  if (ins > 0) {
+    atomicAdd(&q.members, 1u);
+    const uint32_t pos = atomicAdd(&S.tail, 1u);
+    if (pos - head < FW) {
+      atomicAdd(&q.pending, 1u);
+      S.ring_v[pos & (FW - 1)] = v;
+      S.ring_s[pos & (FW - 1)] = (uint16_t)sl;
+    } else {
+      atomicOr(&q.flag, FLAG_RING);  // entry lost: the sample is redone by tier 2
+    }
+  } else if (ins < 0) {
+    atomicOr(&q.flag, FLAG_TABLE);
+  }
+}
+
+__global__ void __launch_bounds__(FG, 2) ic_fused_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
+                                                      SampleCtl* ctl, uint32_t* retry_out, uint32_t chunk,
+                                                      unsigned long long* dbg) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   FusedShared& S = *reinterpret_cast<FusedShared*>(smem_raw);
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -329,9 +376,10 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
     S.exhausted = 0;
   }
   __syncthreads();
-  uint32_t head = 0;
+  uint32_t head = 0, batch_no = 0;
   unsigned long long edges_acc = 0;
   for (;;) {
+    ++batch_no;
     // ---- (1) refill free slots with new samples while the backlog is short
     uint32_t tail = S.tail;
     const uint32_t backlog = tail - head;
@@ -358,6 +406,13 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
         q.pending = 1;
         q.flag = r < 0 ? FLAG_TABLE : 0u;
         q.edges = 0;
+        if (dbg) {
+          unsigned long long tnow;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tnow));
+          q.t_start = tnow;
+          q.levels = 0;
+          q.last_batch = 0xFFFFFFFFu;
+        }
         S.ring_v[(tail + tid) & (FW - 1)] = root;
         S.ring_s[(tail + tid) & (FW - 1)] = sl;
       }
@@ -381,6 +436,7 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
       const uint32_t u = S.ring_v[e];
       const uint16_t sl = S.ring_s[e];
       S.rslot[tid] = sl;
+      if (dbg && atomicExch(&S.slot[sl].last_batch, batch_no) != batch_no) atomicAdd(&S.slot[sl].levels, 1u);
       if (S.slot[sl].flag == 0) {  // rows of failed samples are skipped
         const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
         if (e1 > e0) {
@@ -413,75 +469,83 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
     if ((uint32_t)tid < nb) S.qend[tid] = x + pre;
     head += nb;
     __syncthreads();
-    // ---- (3) sweep the merged quad space
-    int r = -1;
-    uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0, sl_r = 0, sloc_r = 0;
-    unsigned long long q0_r = 0;
-    for (uint32_t base = 0; base < total; base += FU * FG) {
-      unsigned long long qk[FU];
-      uint32_t Tk[FU], mk[FU], slk[FU], sk[FU];
-#pragma unroll
-      for (int k = 0; k < FU; ++k) {
-        const uint32_t j = base + k * FG + tid;
-        mk[k] = 0u;
-        qk[k] = 0ull;
-        Tk[k] = 0u;
-        slk[k] = 0u;
-        sk[k] = 0u;
-        if (j < total) {
-          if (j >= qe) {
-            do {
-              ++r;
-              qe = S.qend[r];
-            } while (j >= qe);
-            nq_r = S.nq[r];
-            qb = qe - nq_r;
-            q0_r = S.q0[r];
-            T_r = S.T[r];
-            wlo_r = S.wlo[r];
-            whi_r = S.whi[r];
-            sl_r = S.rslot[r];
-            sloc_r = S.slot[sl_r].s_local;
-          }
-          const uint32_t li = j - qb;
-          uint32_t m = 0xFu;
-          if (li == 0) m &= 0xFu << wlo_r;
-          if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
-          mk[k] = m;
-          qk[k] = q0_r + li;
-          Tk[k] = T_r;
-          slk[k] = sl_r;
-          sk[k] = sloc_r;
-        }
+    // ---- (3) sweep the merged quad space.  Thread t takes FU = 4 CONSECUTIVE
+    // quads per iteration.  Their row is found by a binary search over the
+    // staged quad ends (no linear walk over small rows).  When the run lies
+    // inside one row (the common case for hub rows) the four Philox calls
+    // share the sample counter and are issued back to back; each quad is
+    // first tested with one 4-way min against T (live edges are rare: ~1 per
+    // expanded row under WC) before the exact per-word test.
+    for (uint32_t base = (uint32_t)tid * FU; base < total; base += FU * FG) {
+      // row r: first row with qend[r] > base
+      uint32_t lo = 0, hi = nb - 1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (S.qend[mid] > base) hi = mid;
+        else lo = mid + 1;
       }
-      uint4 wk[FU];
+      uint32_t r = lo;
+      uint32_t qe = S.qend[r], nq_r = S.nq[r];
+      uint32_t qb = qe - nq_r;
+      if (base + FU <= qe) {
+        // fast path: the whole run is inside row r
+        const uint32_t li = base - qb;
+        const unsigned long long q = S.q0[r] + li;
+        const uint32_t T = S.T[r];
+        const uint32_t sl = S.rslot[r];
+        const uint32_t sloc = S.slot[sl].s_local;
+        const uint64_t sid = R.base + sloc;
+        uint4 wk[FU];
 #pragma unroll
-      for (int k = 0; k < FU; ++k) wk[k] = philox_at(qk[k], R.base + sk[k], TAG_EDGE, K);
+        for (int k = 0; k < FU; ++k) wk[k] = philox_at(q + k, sid, TAG_EDGE, K);
+        uint32_t mk[FU];
 #pragma unroll
+        for (int k = 0; k < FU; ++k) mk[k] = 0xFu;
+        if (li == 0) mk[0] &= 0xFu << S.wlo[r];
+        if (li + FU == nq_r) mk[FU - 1] &= 0xFu >> (3u - S.whi[r]);
+        bool any = false;
+#pragma unroll
+        for (int k = 0; k < FU; ++k) any |= min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= T;
+        if (!any) continue;
+#pragma unroll
+        for (int k = 0; k < FU; ++k) {
+          uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
+                          (wk[k].w <= T ? 8u : 0u);
+          live &= mk[k];
+          while (live) {
+            const int i = __ffs(live) - 1;
+            live &= live - 1;
+            fused_visit(g, R, S, g.nbr[((q + k) << 2) + i], sl, sloc, head);
+          }
+        }
+        continue;
+      }
+      // general path: the run crosses row ends
+#pragma unroll 1
       for (int k = 0; k < FU; ++k) {
-        const uint32_t T = Tk[k];
-        uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
-                        (wk[k].w <= T ? 8u : 0u);
-        live &= mk[k];
+        const uint32_t j = base + k;
+        if (j >= total) break;
+        while (j >= qe) {
+          ++r;
+          qe = S.qend[r];
+          nq_r = S.nq[r];
+        }
+        qb = qe - nq_r;
+        const uint32_t li = j - qb;
+        uint32_t m = 0xFu;
+        if (li == 0) m &= 0xFu << S.wlo[r];
+        if (li == nq_r - 1) m &= 0xFu >> (3u - S.whi[r]);
+        const unsigned long long q = S.q0[r] + li;
+        const uint32_t T = S.T[r];
+        const uint32_t sl = S.rslot[r];
+        const uint32_t sloc = S.slot[sl].s_local;
+        const uint4 w = philox_at(q, R.base + sloc, TAG_EDGE, K);
+        uint32_t live = (w.x <= T ? 1u : 0u) | (w.y <= T ? 2u : 0u) | (w.z <= T ? 4u : 0u) | (w.w <= T ? 8u : 0u);
+        live &= m;
         while (live) {
           const int i = __ffs(live) - 1;
           live &= live - 1;
-          const uint32_t v = g.nbr[(qk[k] << 2) + i];
-          FusedSlot& q = S.slot[slk[k]];
-          const int ins = table_insert(R.keys, R.bits, table_key(sk[k], 0, v));
-          if (ins > 0) {
-            atomicAdd(&q.members, 1u);
-            const uint32_t pos = atomicAdd(&S.tail, 1u);
-            if (pos - head < FW) {
-              atomicAdd(&q.pending, 1u);
-              S.ring_v[pos & (FW - 1)] = v;
-              S.ring_s[pos & (FW - 1)] = (uint16_t)slk[k];
-            } else {
-              atomicOr(&q.flag, FLAG_RING);  // entry lost: the sample is redone by tier 2
-            }
-          } else if (ins < 0) {
-            atomicOr(&q.flag, FLAG_TABLE);
-          }
+          fused_visit(g, R, S, g.nbr[(q << 2) + i], sl, sloc, head);
         }
       }
     }
@@ -492,6 +556,14 @@ __global__ void __launch_bounds__(FG) ic_fused_kernel(GraphView g, uint64_t seed
       FusedSlot& q = S.slot[sl];
       if (atomicSub(&q.pending, 1u) == 1u) {
         const uint32_t f = q.flag;
+        if (dbg) {
+          unsigned long long tnow;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tnow));
+          dbg[4ull * q.s_local + 0] = q.t_start;
+          dbg[4ull * q.s_local + 1] = tnow;
+          dbg[4ull * q.s_local + 2] = q.levels;
+          dbg[4ull * q.s_local + 3] = blockIdx.x | ((unsigned long long)q.edges << 20);
+        }
         if (f == 0u) {
           R.sizes[q.s_local] = q.members;
           edges_acc += q.edges;
@@ -868,8 +940,8 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
     EIM_CUDA(cudaMemsetAsync(R.sizes, 0, count * sizeof(uint32_t), st));
     EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
     EIM_CUDA(cudaEventRecord(ctx->ev0, st));
-    const char* var = getenv("EIM_IC_KERNEL");  // development switch: "group" / "fused" / default "pool"
-    const std::string variant = var ? std::string(var) : std::string("pool");
+    const char* var = getenv("EIM_IC_KERNEL");  // development switch: default "group" / "fused" / "pool"
+    const std::string variant = var ? std::string(var) : std::string("group");
     if (model == EIM_IC && variant == "pool") {
       // task pool capacity from the chunks per sample of earlier rounds
       const double cps = ctx->est_chunks_per_sample > 0 ? ctx->est_chunks_per_sample : 256.0;
@@ -911,8 +983,36 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
       }
       ctx->est_chunks_per_sample = std::max(1.0, (double)used / (double)count);
     } else if (model == EIM_IC && variant == "group") {
-      launch_ic<IC_G, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr,
-                             IC_NG, ~0ull);
+      const char* dbgpath = getenv("EIM_DEBUG_TIMES");
+      unsigned long long* dbgp = nullptr;
+      if (dbgpath) {
+        ctx->stage_c.reserve(count * 48, false, st);
+        dbgp = ctx->stage_c.as<unsigned long long>();
+        EIM_CUDA(cudaMemsetAsync(dbgp, 0, count * 48, st));
+      }
+      EIM_CUDA(cudaMemcpyToSymbolAsync(g_dbg_group, &dbgp, sizeof(dbgp), 0, cudaMemcpyHostToDevice, st));
+      const char* gs = getenv("EIM_IC_G");  // development: group size 256 / 512 / 1024
+      const int gsel = gs ? atoi(gs) : IC_G;
+      if (gsel == 256)
+        launch_ic<256, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr, 1, ~0ull);
+      else if (gsel == 512)
+        launch_ic<512, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr, 1, ~0ull);
+      else
+        launch_ic<1024, false>(ctx, g, seed, R, count, nullptr, IC_W, ctl, ctx->retry_a.as<uint32_t>(), nullptr, 1, ~0ull);
+      if (dbgpath) {
+        std::vector<unsigned long long> hd(count * 6);
+        EIM_CUDA(cudaMemcpyAsync(hd.data(), dbgp, count * 48, cudaMemcpyDeviceToHost, st));
+        EIM_CUDA(cudaStreamSynchronize(st));
+        FILE* f = fopen(dbgpath, "ab");
+        if (f) {
+          const unsigned long long hdr[2] = {first, count};
+          fwrite(hdr, 8, 2, f);
+          fwrite(hd.data(), 8, hd.size(), f);
+          fclose(f);
+        }
+        unsigned long long* nul = nullptr;
+        EIM_CUDA(cudaMemcpyToSymbolAsync(g_dbg_group, &nul, sizeof(nul), 0, cudaMemcpyHostToDevice, st));
+      }
     } else if (model == EIM_IC) {
       const size_t smem = sizeof(FusedShared);
       EIM_CUDA(cudaFuncSetAttribute(ic_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -922,8 +1022,27 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
       blocks = std::max<uint64_t>(1, std::min<uint64_t>(blocks, count));
       // new samples per block per batch: small enough that every block gets a share of the round
       const uint32_t chunk = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(64, count / (blocks * 8)));
+      const char* dbgpath = getenv("EIM_DEBUG_TIMES");
+      unsigned long long* dbg = nullptr;
+      if (dbgpath) {
+        ctx->stage_c.reserve(count * 32, false, st);
+        dbg = ctx->stage_c.as<unsigned long long>();
+        EIM_CUDA(cudaMemsetAsync(dbg, 0, count * 32, st));
+      }
       ic_fused_kernel<<<(uint32_t)blocks, FG, smem, st>>>(g->view, seed, R, count, ctl, ctx->retry_a.as<uint32_t>(),
-                                                          chunk);
+                                                          chunk, dbg);
+      if (dbgpath) {
+        std::vector<unsigned long long> hd(count * 4);
+        EIM_CUDA(cudaMemcpyAsync(hd.data(), dbg, count * 32, cudaMemcpyDeviceToHost, st));
+        EIM_CUDA(cudaStreamSynchronize(st));
+        FILE* f = fopen(dbgpath, "ab");
+        if (f) {
+          const unsigned long long hdr[2] = {first, count};
+          fwrite(hdr, 8, 2, f);
+          fwrite(hd.data(), 8, hd.size(), f);
+          fclose(f);
+        }
+      }
       EIM_CUDA(cudaGetLastError());
       ctx->kernel_launches++;
     } else {
