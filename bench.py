@@ -28,9 +28,26 @@ UNIT = "RRR sets/s"
 GRAPH_SEED = 1
 RUN_SEED = 1
 # ALU roofline of the IC sampler: every examined in-edge costs
-# one Philox4x32-10 word = 10 issue slots (20 IMAD.WIDE + 20 LOP3 per 4
-# words); 148 SMs x 4 schedulers x 32 lanes x 1 instr/clk x 1.965 GHz.
-SM_COUNT, SCHED, LANES, ISSUE_PER_EDGE = 148, 4, 32, 10.0
+# one Philox4x32-10 word; the roof is the Philox word rate of this GPU,
+# measured live by tools/philox_roof (20 IMAD.WIDE per call run at a quarter
+# of the issue rate: ~1.38 calls/clk/SM).  Fallback: the committed
+# measurement in profiles/philox_roof.json.
+PHILOX_PROBE = os.path.join(ROOT, "tools", "philox_roof", "philox_roof")
+
+
+def philox_roof_gwords():
+    try:
+        out = subprocess.run([PHILOX_PROBE], capture_output=True, text=True, timeout=60).stdout
+        vals = [json.loads(l)["words_per_s"] for l in out.splitlines() if l.startswith("{")]
+        if vals:
+            return max(vals) / 1e9, "measured live (tools/philox_roof)"
+    except Exception:
+        pass
+    try:
+        with open(os.path.join(ROOT, "profiles", "philox_roof.json")) as f:
+            return json.load(f)["roof_words_per_s"] / 1e9, "profiles/philox_roof.json (earlier measurement)"
+    except Exception:
+        return 1630.0, "fallback constant"
 
 
 def _peaks():
@@ -39,10 +56,6 @@ def _peaks():
             return json.load(f)
     except Exception:
         return {}
-
-
-def alu_peak_gedges(sm_max_mhz):
-    return SM_COUNT * SCHED * LANES * sm_max_mhz * 1e6 / ISSUE_PER_EDGE / 1e9
 
 
 def workload_desc(cfg_name):
@@ -226,15 +239,14 @@ def main():
     k_ms = sum(s["ms_sample_kernel"] for s in stats)
     k_launch = sum(s["sample_launches"] for s in stats)
     k_edges_local = sum(s["edges_examined"] for s in stats)
-    peaks = _peaks()
-    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
-    peak = alu_peak_gedges(sm_max)
+    peak, peak_src = philox_roof_gwords() if rank == 0 else (1630.0, "")
     achieved = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "latest_traffic.json")
+    traffic = None  # DRAM bytes per sampler launch from the committed ncu --set full capture
+    tpath = os.path.join(ROOT, "profiles", "ncu_sampler.json")
     if os.path.exists(tpath):
         try:
-            traffic = json.load(open(tpath)).get("bytes_per_launch")
+            ls = [l for l in json.load(open(tpath))["launches"] if "dram_bytes" in l]
+            traffic = sum(l["dram_bytes"] for l in ls) / len(ls) if ls else None
         except Exception:
             traffic = None
 
@@ -281,9 +293,11 @@ def main():
                          "sample_kernel": k_ms / args.steps,
                          "select": sum(s["ms_select"] for s in stats) / args.steps,
                          "comm": sum(s["ms_comm"] for s in stats) / args.steps},
-            "roofline": {"bound": "alu", "kernel": "ic_group_kernel (all tiers)", "achieved": achieved, "peak": peak,
-                         "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                         "peak_basis": f"Philox issue roof: 148 SM x 4 sched x 32 lanes x {sm_max:.0f} MHz / 10 instr per edge (DESIGN.md §6)"},
+            "roofline": {"bound": "alu", "kernel": "ic_group_kernel (sampler, all tiers)", "achieved": achieved,
+                         "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
+                         "traffic": traffic,
+                         "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge), "
+                                       + peak_src + "; DESIGN.md §6"},
             "cpu_baseline": cb,
             "e2e": {"value": theta_all / (e2e_ms_step / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": int(off.nbytes + nbr.nbytes), "d2h_bytes_per_step": int(4 * c["k"] + 16),

@@ -79,6 +79,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_probe(force: bool = False) -> str:
+    """tools/philox_roof: the Philox throughput probe bench.py uses as the ALU roof."""
+    src = os.path.join(ROOT, "tools", "philox_roof", "philox_roof.cu")
+    exe = os.path.join(ROOT, "tools", "philox_roof", "philox_roof")
+    hdr = os.path.join(CSRC, "philox.cuh")
+    if force or not os.path.exists(exe) or os.path.getmtime(exe) < max(os.path.getmtime(src), os.path.getmtime(hdr)):
+        subprocess.check_call([_nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "-o", exe, src])
+    return exe
+
+
 if __name__ == "__main__":
     build(force="--force" in sys.argv, verbose="-v" in sys.argv)
     print(LIB)

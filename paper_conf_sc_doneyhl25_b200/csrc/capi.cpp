@@ -17,26 +17,26 @@ void cuda_check(cudaError_t e, const char* what, const char* file, int line) {
   fail(code, std::string(cudaGetErrorString(e)) + " in " + what + " (" + file + ":" + std::to_string(line) + ")");
 }
 
+// Stream-ordered allocation (cudaMallocAsync / cudaFreeAsync): growing a
+// buffer never synchronises the device, so a speculative sampler running on
+// another stream keeps running while the main stream reallocates.
 void DevBuf::reserve(size_t need, bool keep, cudaStream_t st) {
   if (need <= bytes) return;
   size_t nb = std::max(need, bytes + bytes / 2);
   nb = (nb + 255) & ~size_t(255);
   void* q = nullptr;
-  cudaError_t e = cudaMalloc(&q, nb);
+  cudaError_t e = cudaMallocAsync(&q, nb, st);
   if (e != cudaSuccess) {
     cudaGetLastError();
     nb = (need + 255) & ~size_t(255);
-    e = cudaMalloc(&q, nb);
+    e = cudaMallocAsync(&q, nb, st);
     if (e != cudaSuccess) {
       cudaGetLastError();
-      fail(EIM_E_NOMEM, "cudaMalloc of " + std::to_string(nb) + " bytes failed");
+      fail(EIM_E_NOMEM, "cudaMallocAsync of " + std::to_string(nb) + " bytes failed");
     }
   }
-  if (keep && p && bytes) {
-    EIM_CUDA(cudaMemcpyAsync(q, p, bytes, cudaMemcpyDeviceToDevice, st));
-    EIM_CUDA(cudaStreamSynchronize(st));
-  }
-  if (p) cudaFree(p);
+  if (keep && p && bytes) EIM_CUDA(cudaMemcpyAsync(q, p, bytes, cudaMemcpyDeviceToDevice, st));
+  if (p) EIM_CUDA(cudaFreeAsync(p, st));
   p = q;
   bytes = nb;
 }
@@ -91,9 +91,9 @@ void free_ctx_buffers(eim_ctx* c) {
   DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->retry_a, &c->retry_b,
                     &c->tier_tab, &c->tier_queue, &c->tier_gen, &c->C_total, &c->C_work, &c->inv_off,
                     &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
-                    &c->stage_b, &c->stage_c, &c->table, &c->rsizes, &c->rfailed, &c->rfill,
-                    &c->cand, &c->cidx, &c->arena_c, &c->selected, &c->pool, &c->pool_ctl};
+                    &c->stage_b, &c->stage_c, &c->cand, &c->cidx, &c->arena_c, &c->selected};
   for (DevBuf* b : bufs) b->release();
+  for (Round& r : c->rounds) round_release(r);
 }
 
 }  // namespace
@@ -137,6 +137,8 @@ eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint
     try {
       if (c->own_stream) EIM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
       else c->stream = reinterpret_cast<cudaStream_t>(stream);
+      EIM_CUDA(cudaStreamCreateWithFlags(&c->spec_stream, cudaStreamNonBlocking));
+      EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
       EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
       EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
       EIM_CUDA(cudaEventCreate(&c->ev0));
@@ -164,6 +166,9 @@ void eim_destroy(eim_ctx* ctx) {
   cudaFreeHost(ctx->h_pinned);
   cudaEventDestroy(ctx->ev0);
   cudaEventDestroy(ctx->ev1);
+  cudaStreamSynchronize(ctx->spec_stream);
+  cudaStreamDestroy(ctx->spec_stream);
+  cudaStreamDestroy(ctx->aux_stream);
   if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   ctx->magic = 0;
   delete ctx;
@@ -312,7 +317,13 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), st));
     append_sets(ctx, 0, num_sets, ctx->stage_a.as<uint64_t>(), ctx->stage_b.as<uint32_t>(), total);
     hist_sets(ctx, 0, num_sets);
-    greedy(ctx, n, num_sets, k, seeds_out, gains_out);
+    const auto t0 = std::chrono::steady_clock::now();
+    const uint64_t cov = greedy(ctx, n, num_sets, k, seeds_out, gains_out);
+    std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
+    ctx->last_stats.cov = cov;
+    ctx->last_stats.theta = num_sets;
+    ctx->last_stats.arena_elems = total;
+    ctx->last_stats.ms_select = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   });
 }
 

@@ -61,6 +61,20 @@ struct SampleCtl {
 
 struct Comm;  // NCCL communicator wrapper (comm.cpp)
 
+// One sampler launch over sample ids [first, first+count): its membership
+// table and per-sample scratch.  Two of them let the IMM driver sample the
+// next round speculatively while the greedy of the current round runs.
+struct Round {
+  DevBuf table, sizes, failed, edges, fill, retry, excl, ctl;  // ctl: SampleCtl + cancel flag
+  uint64_t first = 0, count = 0, set_base = 0, seed = 0;
+  uint32_t bits = 0;
+  eim_model model = EIM_IC;
+  cudaStream_t stream = nullptr;  // stream the sampler kernel was launched on
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  bool launched = false;
+  bool hist = true;
+};
+
 }  // namespace eim
 
 struct eim_graph {
@@ -87,11 +101,10 @@ struct eim_ctx {
   eim::DevBuf ctl;            // SampleCtl
   eim::DevBuf retry_a, retry_b;
   eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
-  eim::DevBuf table, rsizes, rfailed, rfill;    // per-round membership table + per-sample scratch
+  eim::Round rounds[2];                         // current + speculative sampler rounds
+  cudaStream_t spec_stream = nullptr;           // speculative sampling
+  cudaStream_t aux_stream = nullptr;            // cancel-flag writes
   double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
-  eim::DevBuf pool, pool_ctl;                   // IC task pool (chunk tasks) + its counters
-  double est_chunks_per_sample = 0;
-  uint64_t pool_dirty = 0, pool_cap_hint = 0;
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;
@@ -120,9 +133,20 @@ struct SampleResult {
   double kernel_ms = 0;
 };
 // Samples ids [first, first+count) into ctx->arena; set index = id - set_base.
-// Histogram into C when hist is true.
+// Histogram into C when hist is true.  (= round_launch + round_finalize)
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
                           uint64_t first, uint64_t count, uint64_t set_base, bool hist);
+// Launch the sampler for ids [first, first+count) into rd on stream st (no
+// host synchronisation).  spare_sm_slot: leave one block slot per SM free
+// (for a concurrent greedy kernel).
+void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first,
+                  uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot);
+// Wait for rd, redo what overflowed, and append its first `use` sets to the
+// arena (sample-id order) with their histogram.
+SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use);
+// Stop a launched speculative round and wait for it.
+void round_cancel(eim_ctx* ctx, Round& rd);
+void round_release(Round& rd);
 void arena_reset(eim_ctx* ctx);
 void ensure_sets(eim_ctx* ctx, uint64_t num_sets);
 uint64_t arena_cursor(eim_ctx* ctx);

@@ -7,6 +7,7 @@
 // the shares are all-gathered over NCCL in rank (= sample-id) order and the
 // greedy runs replicated on identical data, so results equal the 1-GPU run.
 #include <chrono>
+#include <cstdlib>
 #include <cmath>
 #include <cstring>
 
@@ -49,15 +50,6 @@ struct Exchange {
 void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t R, uint64_t R_new,
                   eim_stats* st, Exchange& ex) {
   const auto t0 = clk::now();
-  if (ctx->world == 1) {
-    SampleResult r = sample_range(ctx, g, model, seed, R, R_new - R, 0, true);
-    st->edges_examined += r.edges;
-    st->tier2_samples += r.tier2;
-    st->sample_launches += r.launches;
-    st->ms_sample_kernel += r.kernel_ms;
-    st->ms_sample += ms_since(t0);
-    return;
-  }
   cudaStream_t s = ctx->stream;
   uint64_t lo, hi;
   eim_shard_range(R, R_new - R, ctx->rank, ctx->world, &lo, &hi);
@@ -107,6 +99,82 @@ void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   st->ms_sample += ms_since(t0);
 }
 
+// Supplies the sets of sample ids [|R|, to) to the arena.  On one GPU the
+// next round's ids are sampled SPECULATIVELY on a second stream while the
+// current round's greedy runs (sample ids are fixed labels, so a speculative
+// set is exactly the set the next round needs); a round that turns out not
+// to be needed is cancelled.  This hides each round's sampling tail -- the
+// last long reverse-BFS chains, which keep only a few SMs busy -- behind
+// useful work.
+class RoundSampler {
+ public:
+  RoundSampler(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, eim_stats* st)
+      : ctx_(ctx), g_(g), model_(model), seed_(seed), st_(st) {
+    speculate_ = ctx->world == 1 && std::getenv("EIM_NO_SPECULATION") == nullptr;
+  }
+  ~RoundSampler() {
+    ex_.counts.release();
+    ex_.offs_recv.release();
+    ex_.mem_recv.release();
+  }
+
+  void grow(uint64_t& R, uint64_t to) {
+    if (to <= R) return;
+    const auto t0 = clk::now();
+    if (ctx_->world > 1) {
+      sample_round(ctx_, g_, model_, seed_, R, to, st_, ex_);
+      R = to;
+      return;
+    }
+    if (spec_ && spec_->first == R) {
+      const uint64_t use = std::min<uint64_t>(spec_->count, to - R);
+      account(round_finalize(ctx_, g_, *spec_, use));
+      R += use;
+      spec_ = nullptr;
+    } else {
+      cancel();
+    }
+    if (to > R) {
+      Round& rd = free_round();
+      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, ctx_->stream, false);
+      account(round_finalize(ctx_, g_, rd, to - R));
+      R = to;
+    }
+    st_->ms_sample += ms_since(t0);
+  }
+
+  void speculate(uint64_t R, uint64_t to) {
+    if (!speculate_ || to <= R || spec_) return;
+    Round& rd = free_round();
+    round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, ctx_->spec_stream, true);
+    spec_ = &rd;
+  }
+
+  void cancel() {
+    if (spec_) {
+      round_cancel(ctx_, *spec_);
+      spec_ = nullptr;
+    }
+  }
+
+ private:
+  Round& free_round() { return spec_ == &ctx_->rounds[0] ? ctx_->rounds[1] : ctx_->rounds[0]; }
+  void account(const SampleResult& r) {
+    st_->edges_examined += r.edges;
+    st_->tier2_samples += r.tier2;
+    st_->sample_launches += r.launches;
+    st_->ms_sample_kernel += r.kernel_ms;
+  }
+  eim_ctx* ctx_;
+  const eim_graph* g_;
+  eim_model model_;
+  uint64_t seed_;
+  eim_stats* st_;
+  Exchange ex_;
+  bool speculate_ = false;
+  Round* spec_ = nullptr;
+};
+
 }  // namespace
 
 void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
@@ -124,36 +192,37 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   arena_reset(ctx);
   ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
   EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
-  Exchange ex;
+  RoundSampler sampler(ctx, g, model, seed, st);
   std::vector<uint32_t> S(k);
   uint64_t R = 0, cov = 0;
   uint64_t R_selected = UINT64_MAX;  // |R| the last NodeSelection ran on
   double LB = 1.0;
-  for (uint32_t i = 1; (double)i < p.log2n; ++i) {
-    const uint64_t theta_i = (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n);
-    if (theta_i > R) {
-      sample_round(ctx, g, model, seed, R, theta_i, st, ex);
-      R = theta_i;
+  auto theta_round = [&](uint32_t i) { return (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n); };
+  try {
+    for (uint32_t i = 1; (double)i < p.log2n; ++i) {
+      sampler.grow(R, theta_round(i));
+      if ((double)(i + 1) < p.log2n) sampler.speculate(R, theta_round(i + 1));
+      const auto ts = clk::now();
+      cov = greedy(ctx, n, R, k, S.data(), nullptr);
+      st->ms_select += ms_since(ts);
+      R_selected = R;
+      if (st->rounds < 64) {
+        st->theta_i[st->rounds] = R;
+        st->cov_i[st->rounds] = cov;
+      }
+      st->rounds++;
+      if ((double)cov * std::ldexp(1.0, (int)i) >= (1.0 + p.eps_p) * (double)R) {
+        LB = ((double)n * (double)cov) / ((1.0 + p.eps_p) * (double)R);
+        break;
+      }
     }
-    const auto ts = clk::now();
-    cov = greedy(ctx, n, R, k, S.data(), nullptr);
-    st->ms_select += ms_since(ts);
-    R_selected = R;
-    if (st->rounds < 64) {
-      st->theta_i[st->rounds] = R;
-      st->cov_i[st->rounds] = cov;
-    }
-    st->rounds++;
-    if ((double)cov * std::ldexp(1.0, (int)i) >= (1.0 + p.eps_p) * (double)R) {
-      LB = ((double)n * (double)cov) / ((1.0 + p.eps_p) * (double)R);
-      break;
-    }
-  }
-  st->lb = LB;
-  const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
-  if (theta > R) {
-    sample_round(ctx, g, model, seed, R, theta, st, ex);
-    R = theta;
+    st->lb = LB;
+    const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
+    sampler.grow(R, theta);
+    sampler.cancel();
+  } catch (...) {
+    sampler.cancel();
+    throw;
   }
   if (R != R_selected) {  // NodeSelection is deterministic: reuse the last run on the same R
     const auto ts = clk::now();
@@ -163,14 +232,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   std::memcpy(seeds_out, S.data(), (size_t)k * sizeof(uint32_t));
   st->theta = R;
   st->cov = cov;
-  st->arena_elems = 0;
-  {
-    // arena elements of all sets = sum of C_total
-    st->arena_elems = arena_cursor(ctx);
-  }
-  ex.counts.release();
-  ex.offs_recv.release();
-  ex.mem_recv.release();
+  st->arena_elems = arena_cursor(ctx);
   if (theta_out) *theta_out = R;
   if (spread_out) *spread_out = (double)n * (double)cov / (double)R;
   st->kernel_launches = ctx->kernel_launches - launches0;

@@ -18,6 +18,10 @@
 //      pick is the lowest unselected vertex id (R10).
 #include <cooperative_groups.h>
 
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+
 #include <cub/cub.cuh>
 
 #include "eim_internal.h"
@@ -29,7 +33,7 @@ namespace eim {
 namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
-constexpr int GB = 256;  // threads per block of the greedy kernel
+constexpr int GB = 256;  // threads per block of the greedy kernel (one block per SM: fits next to a running sampler)
 
 __global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t* __restrict__ flags) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -125,7 +129,14 @@ struct GreedyArgs {
   uint32_t* zc;                 // cursor of the lowest possibly-unselected id
   uint32_t* seeds;
   unsigned long long* gains;
+  unsigned long long* dbg;      // development: per-pick timestamps (nullable)
 };
+
+__device__ __forceinline__ unsigned long long gtimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   cg::grid_group grid = cg::this_grid();
@@ -136,6 +147,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   const uint64_t warp = ((uint64_t)blockIdx.x * GB + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * GB) >> 5;
   for (uint32_t j = 0; j < a.k; ++j) {
+    if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j] = gtimer_ns();
     // ---- argmax over this block's slice
     unsigned long long km = 0;
     for (uint32_t i = blockIdx.x * GB + threadIdx.x; i < nc4; i += gridDim.x * GB) {
@@ -149,6 +161,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
     km = block_max(km, red);
     if (threadIdx.x == 0) a.blockmax[blockIdx.x] = km;
     grid.sync();
+    if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 1] = gtimer_ns();
     km = 0;
     for (uint32_t b = threadIdx.x; b < gridDim.x; b += GB) km = umax64(km, a.blockmax[b]);
     km = block_max(km, red);
@@ -182,6 +195,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         for (uint32_t t = lane; t < L; t += 32) atomicSub(&a.W[a.arena_c[st + t]], 1u);
       }
     }
+    if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 2] = gtimer_ns();
     grid.sync();
   }
 }
@@ -244,7 +258,9 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   EIM_CUDA(cudaMemsetAsync(ctx->selected.p, 0, (uint64_t)n + 4, st));
   int per_sm = 0;
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
-  uint32_t blocks = (uint32_t)std::max(1, std::min(per_sm, 4)) * ctx->sm_count;
+  const char* gbe = getenv("EIM_GREEDY_BPSM");  // development: blocks per SM of the greedy kernel
+  const int bpsm = gbe ? atoi(gbe) : 1;
+  uint32_t blocks = (uint32_t)std::max(1, std::min(per_sm, bpsm)) * ctx->sm_count;
   ctx->best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
   uint32_t* zc = reinterpret_cast<uint32_t*>(ctx->best.as<unsigned long long>() + blocks);
   EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
@@ -264,9 +280,25 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   a.zc = zc;
   a.seeds = ctx->seeds.as<uint32_t>();
   a.gains = ctx->gains.as<unsigned long long>();
+  a.dbg = nullptr;
+  const char* gdbg = getenv("EIM_DEBUG_GREEDY");
+  if (gdbg) {
+    ctx->stage_a.reserve((uint64_t)k * 24 + 64, false, st);
+    a.dbg = ctx->stage_a.as<unsigned long long>();
+  }
   void* args[] = {&a};
   EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
   ctx->kernel_launches += 9;
+  if (gdbg) {
+    std::vector<unsigned long long> hd((size_t)k * 3);
+    EIM_CUDA(cudaMemcpyAsync(hd.data(), a.dbg, (size_t)k * 24, cudaMemcpyDeviceToHost, st));
+    EIM_CUDA(cudaStreamSynchronize(st));
+    FILE* f = fopen(gdbg, "ab");
+    if (f) {
+      fwrite(hd.data(), 8, hd.size(), f);
+      fclose(f);
+    }
+  }
   std::vector<unsigned long long> g(k);
   EIM_CUDA(cudaMemcpyAsync(seeds_out, ctx->seeds.p, (uint64_t)k * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaMemcpyAsync(g.data(), ctx->gains.p, (uint64_t)k * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));

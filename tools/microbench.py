@@ -50,5 +50,26 @@ def main():
     eim.eim_destroy(ctx)
 
 
+
+
+def greedy_bench():
+    """select_seeds on a GPU-sampled C2 arena of 101294 sets (the last IMM round)."""
+    c = inputs.CONFIGS["C2"]
+    off, nbr = inputs.config_graph("C2")
+    ctx = eim.eim_create(0)
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    o, m = eim.eim_sample_rrr(ctx, g, "IC", 1, 0, 101294)
+    for _ in range(2):
+        eim.eim_select_seeds(ctx, c["n"], o, m, c["k"])
+    times = []
+    for _ in range(5):
+        eim.eim_select_seeds(ctx, c["n"], o, m, c["k"])
+        times.append(eim.eim_get_stats(ctx)["ms_select"])
+    print("greedy", json.dumps(dict(k=c["k"], sets=101294, members=int(m.size), ms=sorted(times))))
+
+
 if __name__ == "__main__":
-    main()
+    if "--greedy" in sys.argv:
+        greedy_bench()
+    else:
+        main()
