@@ -137,7 +137,8 @@ eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint
     try {
       if (c->own_stream) EIM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
       else c->stream = reinterpret_cast<cudaStream_t>(stream);
-      EIM_CUDA(cudaStreamCreateWithFlags(&c->spec_stream, cudaStreamNonBlocking));
+      EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[0], cudaStreamNonBlocking));
+      EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
       EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
       EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
       EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
@@ -166,8 +167,10 @@ void eim_destroy(eim_ctx* ctx) {
   cudaFreeHost(ctx->h_pinned);
   cudaEventDestroy(ctx->ev0);
   cudaEventDestroy(ctx->ev1);
-  cudaStreamSynchronize(ctx->spec_stream);
-  cudaStreamDestroy(ctx->spec_stream);
+  for (cudaStream_t rs : ctx->rstream) {
+    cudaStreamSynchronize(rs);
+    cudaStreamDestroy(rs);
+  }
   cudaStreamDestroy(ctx->aux_stream);
   if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   ctx->magic = 0;

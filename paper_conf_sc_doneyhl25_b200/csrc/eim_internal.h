@@ -57,6 +57,8 @@ struct SampleCtl {
   unsigned long long retry_count;
   unsigned long long edges;
   unsigned long long arena_fail;
+  unsigned long long active;  // samples in progress (tier-1 tail hand-off)
+  unsigned long long pad;
 };
 
 struct Comm;  // NCCL communicator wrapper (comm.cpp)
@@ -69,8 +71,10 @@ struct Round {
   uint64_t first = 0, count = 0, set_base = 0, seed = 0;
   uint32_t bits = 0;
   eim_model model = EIM_IC;
-  cudaStream_t stream = nullptr;  // stream the sampler kernel was launched on
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  cudaStream_t stream = nullptr;  // stream the sampler kernels were launched on
+  static constexpr int MAX_LAUNCH = 8;
+  cudaEvent_t ev[2 * MAX_LAUNCH] = {};  // start/stop of every sampler launch of the round
+  int nlaunch = 0;
   bool launched = false;
   bool hist = true;
 };
@@ -102,7 +106,7 @@ struct eim_ctx {
   eim::DevBuf retry_a, retry_b;
   eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
   eim::Round rounds[2];                         // current + speculative sampler rounds
-  cudaStream_t spec_stream = nullptr;           // speculative sampling
+  cudaStream_t rstream[2] = {};                 // sampler streams of rounds[0], rounds[1]
   cudaStream_t aux_stream = nullptr;            // cancel-flag writes
   double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
   // per-graph vectors
@@ -146,6 +150,10 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use);
 // Stop a launched speculative round and wait for it.
 void round_cancel(eim_ctx* ctx, Round& rd);
+// Let a launched round take no new sample ids (its running samples finish);
+// round_resume relaunches it on st, continuing with the remaining ids.
+void round_pause(eim_ctx* ctx, Round& rd);
+void round_resume(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st);
 void round_release(Round& rd);
 void arena_reset(eim_ctx* ctx);
 void ensure_sets(eim_ctx* ctx, uint64_t num_sets);

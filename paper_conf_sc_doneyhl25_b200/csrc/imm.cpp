@@ -100,17 +100,21 @@ void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 }
 
 // Supplies the sets of sample ids [|R|, to) to the arena.  On one GPU the
-// next round's ids are sampled SPECULATIVELY on a second stream while the
-// current round's greedy runs (sample ids are fixed labels, so a speculative
-// set is exactly the set the next round needs); a round that turns out not
-// to be needed is cancelled.  This hides each round's sampling tail -- the
-// last long reverse-BFS chains, which keep only a few SMs busy -- behind
-// useful work.
+// next round's ids [to, next_to) are launched SPECULATIVELY on a second
+// stream right behind the current round's launch: its blocks take the SMs
+// that the current round's tail (its last, longest reverse-BFS chains)
+// leaves idle.  While the greedy of the current round runs, the speculative
+// round is paused (it takes no new ids, so the greedy has the GPU); it is
+// resumed when its ids are needed, or cancelled when they are not.  Sample
+// ids are fixed labels, so a speculative set is exactly the set the next
+// round needs and results are unchanged.
 class RoundSampler {
  public:
   RoundSampler(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, eim_stats* st)
       : ctx_(ctx), g_(g), model_(model), seed_(seed), st_(st) {
-    speculate_ = ctx->world == 1 && std::getenv("EIM_NO_SPECULATION") == nullptr;
+    // opt-in (EIM_SPECULATE=1): measured on C2 the speculative round slows the
+    // current round's critical chains as much as it fills their idle SMs
+    speculate_ = ctx->world == 1 && std::getenv("EIM_SPECULATE") != nullptr;
   }
   ~RoundSampler() {
     ex_.counts.release();
@@ -118,7 +122,8 @@ class RoundSampler {
     ex_.mem_recv.release();
   }
 
-  void grow(uint64_t& R, uint64_t to) {
+  // make sets [R, to) final; speculate [to, next_to)
+  void grow(uint64_t& R, uint64_t to, uint64_t next_to) {
     if (to <= R) return;
     const auto t0 = clk::now();
     if (ctx_->world > 1) {
@@ -126,28 +131,34 @@ class RoundSampler {
       R = to;
       return;
     }
+    Round* cur = nullptr;
     if (spec_ && spec_->first == R) {
-      const uint64_t use = std::min<uint64_t>(spec_->count, to - R);
-      account(round_finalize(ctx_, g_, *spec_, use));
-      R += use;
+      cur = spec_;
       spec_ = nullptr;
+      round_resume(ctx_, g_, *cur, stream_of(*cur));
     } else {
       cancel();
+      cur = &ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, *cur, stream_of(*cur), false);
     }
-    if (to > R) {
-      Round& rd = free_round();
-      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, ctx_->stream, false);
+    const uint64_t cur_end = R + cur->count;
+    if (speculate_ && next_to > cur_end) {
+      Round& nx = (cur == &ctx_->rounds[0]) ? ctx_->rounds[1] : ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, cur_end, next_to - cur_end, 0, true, nx, stream_of(nx), true);
+      spec_ = &nx;
+    }
+    const uint64_t use = std::min<uint64_t>(cur->count, to - R);
+    account(round_finalize(ctx_, g_, *cur, use));
+    R += use;
+    if (to > R) {  // the speculative range was shorter than needed: sample the rest now
+      cancel();
+      Round& rd = ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, stream_of(rd), false);
       account(round_finalize(ctx_, g_, rd, to - R));
       R = to;
     }
+    if (spec_) round_pause(ctx_, *spec_);
     st_->ms_sample += ms_since(t0);
-  }
-
-  void speculate(uint64_t R, uint64_t to) {
-    if (!speculate_ || to <= R || spec_) return;
-    Round& rd = free_round();
-    round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, ctx_->spec_stream, true);
-    spec_ = &rd;
   }
 
   void cancel() {
@@ -158,7 +169,7 @@ class RoundSampler {
   }
 
  private:
-  Round& free_round() { return spec_ == &ctx_->rounds[0] ? ctx_->rounds[1] : ctx_->rounds[0]; }
+  cudaStream_t stream_of(const Round& rd) const { return &rd == &ctx_->rounds[0] ? ctx_->rstream[0] : ctx_->rstream[1]; }
   void account(const SampleResult& r) {
     st_->edges_examined += r.edges;
     st_->tier2_samples += r.tier2;
@@ -200,8 +211,8 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   auto theta_round = [&](uint32_t i) { return (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n); };
   try {
     for (uint32_t i = 1; (double)i < p.log2n; ++i) {
-      sampler.grow(R, theta_round(i));
-      if ((double)(i + 1) < p.log2n) sampler.speculate(R, theta_round(i + 1));
+      const uint64_t next = (double)(i + 1) < p.log2n ? theta_round(i + 1) : 0;
+      sampler.grow(R, theta_round(i), next);
       const auto ts = clk::now();
       cov = greedy(ctx, n, R, k, S.data(), nullptr);
       st->ms_select += ms_since(ts);
@@ -218,7 +229,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
     }
     st->lb = LB;
     const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
-    sampler.grow(R, theta);
+    sampler.grow(R, theta, 0);
     sampler.cancel();
   } catch (...) {
     sampler.cancel();

@@ -44,9 +44,11 @@ constexpr int IC_NG = 1;           // groups per block
 constexpr int IC_U = 2;            // consecutive quads per thread per sweep iteration
 
 // ---------------------------------------------------------------- table
-// key = ((s_local + 1) | tier << 31) << 32 | v ;  0 = empty slot.
+// key = ((s_local + 1) | tier << 30) << 32 | v ;  0 = empty slot.  tier =
+// attempt number of the sample (0, 1, 2): the scatter keeps only the keys of
+// the attempt that succeeded.
 __device__ __forceinline__ unsigned long long table_key(uint32_t s_local, uint32_t tier, uint32_t v) {
-  return ((unsigned long long)((s_local + 1u) | (tier << 31)) << 32) | (unsigned long long)v;
+  return ((unsigned long long)((s_local + 1u) | (tier << 30)) << 32) | (unsigned long long)v;
 }
 
 __device__ __forceinline__ uint32_t table_hash(unsigned long long key, uint32_t bits) {
@@ -116,15 +118,15 @@ __device__ __forceinline__ uint32_t group_incl_scan(uint32_t x, int gtid, int gi
   }
 }
 
-enum : uint32_t { FLAG_RING = 1u, FLAG_TABLE = 2u, FLAG_CANCEL = 4u };
+enum : uint32_t { FLAG_RING = 1u, FLAG_TABLE = 2u, FLAG_CANCEL = 4u, FLAG_HANDOFF = 8u };
 
 struct RoundView {
   unsigned long long* keys;
   uint32_t bits;
   uint32_t* sizes;               // [count] members per sample (s_local)
-  uint8_t* failed;               // [count] 1 = tier-1 attempt abandoned (its tier-0 keys are ignored)
+  uint8_t* failed;               // [count] attempt (tier) whose keys are the sample's members
   unsigned long long* edges;     // [count] examined in-edges (IC) / walk steps (LT) per sample
-  const unsigned int* cancel;    // nonzero: stop (a speculative round that is not needed)
+  const unsigned int* cancel;    // [0] cancel (round not needed), [1] pause (take no new ids)
   uint64_t base;                 // sample id of s_local = 0
 };
 
@@ -156,7 +158,8 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
                                                     uint32_t s_local, uint32_t tier, uint32_t* ring, uint32_t W,
                                                     const RingRows* rr, uint32_t* live_v, GroupRows<G>& rw,
                                                     GroupCtl& gc, int gtid, int gi, unsigned long long& se,
-                                                    uint32_t& size) {
+                                                    uint32_t& size, const SampleCtl* ctl, uint64_t count,
+                                                    uint32_t handoff) {
   const uint64_t s = R.base + s_local;
   uint32_t head = 0;
   // visit v: table insert; a new member is appended to the ring (with its row)
@@ -291,6 +294,12 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
     // ---- visit the parked live neighbours, one per thread
     const uint32_t nl = min(*(volatile uint32_t*)&gc.nlive, LIVE_CAP);
     for (uint32_t t = gtid; t < nl; t += G) visit(live_v[t]);
+    // tail hand-off: once the launch has no new ids left and only a few
+    // samples are still running (the long chains), give this one up; the
+    // host redoes it with a whole SM per sample (tier 2)
+    if (handoff && gtid == 0 && *(volatile const unsigned long long*)&ctl->ticket >= count &&
+        *(volatile const unsigned long long*)&ctl->active <= handoff)
+      atomicOr(&gc.flag, FLAG_HANDOFF);
     gsync<G>(gi);
   }
 }
@@ -299,11 +308,12 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
 // over the contiguous ids [0, count).  tier 2 (GLOBAL_RING = true): ring of W
 // entries per group slot in global memory, over a list of failed ids.
 template <int G, bool GLOBAL_RING>
-__global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
+__global__ void __launch_bounds__(G, (G >= 1024 ? 1 : (G >= 512 ? 2 : 6))) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
                                                                         uint64_t count,
                                                                         const uint32_t* __restrict__ ids,
                                                                         uint32_t W, SampleCtl* ctl,
-                                                                        uint32_t* retry_out, uint32_t* gring) {
+                                                                        uint32_t* retry_out, uint32_t* gring,
+                                                                        uint32_t tier, uint32_t handoff) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int gi = threadIdx.x / G, gtid = threadIdx.x % G;
   const size_t per_group = sizeof(GroupCtl) + sizeof(GroupRows<G>) + 4 * LIVE_CAP + (GLOBAL_RING ? 0 : (size_t)20 * W);
@@ -322,30 +332,38 @@ __global__ void __launch_bounds__(G) ic_group_kernel(GraphView g, uint64_t seed,
     rows_smem.T = reinterpret_cast<uint32_t*>(dyn + 16ull * W);
   }
   const RingRows* rr = GLOBAL_RING ? nullptr : &rows_smem;
-  const uint32_t tier = GLOBAL_RING ? 1u : 0u;
   const PhiloxKey K = philox_key(seed);
   unsigned long long edges_acc = 0;
   for (;;) {
     if (gtid == 0) {
-      const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
-      const bool stop = t >= count || *(volatile const unsigned int*)R.cancel;
+      // cancelled or paused: take no new id (a resumed launch continues the ticket)
+      const volatile unsigned int* cp = R.cancel;
+      bool stop = cp[0] || cp[1];
+      unsigned long long t = 0;
+      if (!stop) {
+        t = atomicAdd(&ctl->ticket, 1ull);
+        stop = t >= count;
+      }
       gc.s_local = stop ? 0xFFFFFFFFu : (ids ? ids[t] : (uint32_t)t);
+      if (!stop) atomicAdd(&ctl->active, 1ull);
     }
     gsync<G>(gi);
     const uint32_t s_local = gc.s_local;
     if (s_local == 0xFFFFFFFFu) break;
     unsigned long long se = 0;
     uint32_t size = 0;
-    const uint32_t flag = ic_group_sample<G, IC_U>(g, K, R, s_local, tier, ring, W, rr, live_v, rw, gc, gtid, gi, se, size);
+    const uint32_t flag = ic_group_sample<G, IC_U>(g, K, R, s_local, tier, ring, W, rr, live_v, rw, gc, gtid, gi, se,
+                                                       size, ctl, count, handoff);
     if (gtid == 0) {
       if (flag == 0) {
         R.sizes[s_local] = size;
       } else if (flag & FLAG_TABLE) {
         atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);  // table too full: host redoes the round
-      } else if (flag & FLAG_RING) {
-        R.failed[s_local] = 1;
+      } else if (flag & (FLAG_RING | FLAG_HANDOFF)) {
+        R.failed[s_local] = (uint8_t)(tier + 1);  // the next attempt's keys will be the members
         retry_out[atomicAdd(&ctl->retry_count, 1ull)] = s_local;
       }
+      atomicAdd(&ctl->active, ~0ull);  // -1
     }
     if (flag == 0) {
       edges_acc += se;
@@ -370,8 +388,10 @@ __global__ void __launch_bounds__(256) lt_kernel(GraphView g, uint64_t seed, Rou
   const PhiloxKey K = philox_key(seed);
   unsigned long long edges_acc = 0;
   for (;;) {
+    const volatile unsigned int* cp = R.cancel;
+    if (cp[0] || cp[1]) break;  // cancelled or paused
     const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
-    if (t >= count || *(volatile const unsigned int*)R.cancel) break;
+    if (t >= count) break;
     const uint32_t s_local = (uint32_t)t;
     const uint64_t s = R.base + s_local;
     uint32_t u = draw_root(s, g.n, K);
@@ -431,10 +451,10 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
     const unsigned long long k = keys[i];
     if (k == 0ull) continue;
     const uint32_t hi = (uint32_t)(k >> 32);
-    const uint32_t tier = hi >> 31;
-    const uint32_t s_local = (hi & 0x7FFFFFFFu) - 1u;
+    const uint32_t tier = hi >> 30;
+    const uint32_t s_local = (hi & 0x3FFFFFFFu) - 1u;
     if (s_local >= use) continue;                // speculative samples beyond the ones kept
-    if (tier == 0 && failed[s_local]) continue;  // abandoned tier-1 attempt; redone under tier-2 keys
+    if (tier != failed[s_local]) continue;       // an abandoned attempt of a sample that was redone
     const uint32_t v = (uint32_t)k;
     const uint32_t p = atomicAdd(&fill[s_local], 1u);
     arena[set_start[set_index0 + s_local] + p] = v;
@@ -443,7 +463,9 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
 }
 
 constexpr uint32_t IC_W = 1024;    // shared-memory frontier ring per group
-constexpr int IC_G2 = 512;         // tier 2 (global ring of capacity >= n)
+constexpr int IC_G2 = 1024;        // tier 2: a whole SM per sample (tail hand-off and ring overflow)
+constexpr uint32_t IC_W2 = 4096;   // tier-2 shared-memory ring
+constexpr int IC_G3 = 512;         // tier 3: global ring of capacity >= n (never fails)
 
 template <int G, bool GR>
 size_t ic_smem_per_group(uint32_t W) {
@@ -477,16 +499,17 @@ void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
 void round_release(Round& rd) {
   DevBuf* b[] = {&rd.table, &rd.sizes, &rd.failed, &rd.edges, &rd.fill, &rd.retry, &rd.excl, &rd.ctl};
   for (DevBuf* x : b) x->release();
-  if (rd.ev0) cudaEventDestroy(rd.ev0);
-  if (rd.ev1) cudaEventDestroy(rd.ev1);
-  rd.ev0 = rd.ev1 = nullptr;
+  for (cudaEvent_t& e : rd.ev) {
+    if (e) cudaEventDestroy(e);
+    e = nullptr;
+  }
   rd.launched = false;
 }
 
 template <int G, bool GR>
 static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, const RoundView& R, uint64_t count,
                       const uint32_t* ids, uint32_t W, SampleCtl* ctl, uint32_t* retry_out, uint32_t* gring,
-                      uint64_t max_blocks, cudaStream_t st, bool spare_sm_slot) {
+                      uint64_t max_blocks, cudaStream_t st, bool spare_sm_slot, uint32_t tier, uint32_t handoff) {
   const size_t smem = ic_smem_per_group<G, GR>(W);
   auto kern = ic_group_kernel<G, GR>;
   EIM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -496,9 +519,18 @@ static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, const Rou
   if (spare_sm_slot && per_sm > 1) per_sm -= 1;
   uint64_t blocks = (uint64_t)per_sm * ctx->sm_count;
   blocks = std::max<uint64_t>(1, std::min<uint64_t>(std::min<uint64_t>(blocks, count), max_blocks));
-  kern<<<(uint32_t)blocks, G, smem, st>>>(g->view, seed, R, count, ids, W, ctl, retry_out, gring);
+  kern<<<(uint32_t)blocks, G, smem, st>>>(g->view, seed, R, count, ids, W, ctl, retry_out, gring, tier, handoff);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
+}
+
+// Tail hand-off threshold of tier 1 (samples still running when the launch
+// has no ids left), off by default: measured on C2 it did not shorten the
+// rounds (a restarted chain costs about what it had left).  EIM_HANDOFF=<n>
+// enables it for experiments.
+static uint32_t handoff_threshold(eim_ctx*) {
+  const char* e = std::getenv("EIM_HANDOFF");
+  return e ? (uint32_t)std::atoi(e) : 0u;
 }
 
 static RoundView round_view(Round& rd) {
@@ -507,43 +539,64 @@ static RoundView round_view(Round& rd) {
                    reinterpret_cast<const unsigned int*>(rd.ctl.as<SampleCtl>() + 1), rd.first};
 }
 
-// memsets + tier-1 launch of rd's range on stream st
-static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
-  const uint64_t count = rd.count;
-  rd.table.reserve(8ull << rd.bits, false, st);
+// one tier-1 sampler launch over rd's remaining ids, bracketed by events
+static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
+  if (rd.nlaunch >= Round::MAX_LAUNCH) fail(EIM_E_STATE, "too many sampler launches in one round");
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
-  EIM_CUDA(cudaMemsetAsync(rd.table.p, 0, 8ull << rd.bits, st));
-  EIM_CUDA(cudaMemsetAsync(rd.failed.p, 0, count, st));
-  EIM_CUDA(cudaMemsetAsync(rd.sizes.p, 0, count * sizeof(uint32_t), st));
-  EIM_CUDA(cudaMemsetAsync(rd.edges.p, 0, count * sizeof(unsigned long long), st));
-  EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl) + 16, st));
   const RoundView R = round_view(rd);
-  EIM_CUDA(cudaEventRecord(rd.ev0, st));
+  EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch], st));
   if (rd.model == EIM_IC) {
-    launch_ic<IC_G, false>(ctx, g, rd.seed, R, count, nullptr, IC_W, ctl, rd.retry.as<uint32_t>(), nullptr, ~0ull,
-                           st, spare_sm_slot);
+    launch_ic<IC_G, false>(ctx, g, rd.seed, R, rd.count, nullptr, IC_W, ctl, rd.retry.as<uint32_t>(), nullptr,
+                           ~0ull, st, spare_sm_slot, 0, handoff_threshold(ctx));
   } else {
     int per_sm = 0;
     EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel, 256, 0));
     if (spare_sm_slot && per_sm > 1) per_sm -= 1;
-    uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (count + 255) / 256);
-    lt_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(g->view, rd.seed, R, count, ctl);
+    uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
+    lt_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(g->view, rd.seed, R, rd.count, ctl);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
   }
-  EIM_CUDA(cudaEventRecord(rd.ev1, st));
+  EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch + 1], st));
+  rd.nlaunch++;
   rd.stream = st;
   rd.launched = true;
+}
+
+// memsets + first tier-1 launch of rd's range on stream st
+static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
+  const uint64_t count = rd.count;
+  rd.table.reserve(8ull << rd.bits, false, st);
+  EIM_CUDA(cudaMemsetAsync(rd.table.p, 0, 8ull << rd.bits, st));
+  EIM_CUDA(cudaMemsetAsync(rd.failed.p, 0, count, st));
+  EIM_CUDA(cudaMemsetAsync(rd.sizes.p, 0, count * sizeof(uint32_t), st));
+  EIM_CUDA(cudaMemsetAsync(rd.edges.p, 0, count * sizeof(unsigned long long), st));
+  EIM_CUDA(cudaMemsetAsync(rd.ctl.p, 0, sizeof(SampleCtl) + 16, st));
+  rd.nlaunch = 0;
+  round_kernel(ctx, g, rd, st, spare_sm_slot);
+}
+
+static unsigned int* round_flags(Round& rd) { return reinterpret_cast<unsigned int*>(rd.ctl.as<SampleCtl>() + 1); }
+
+void round_pause(eim_ctx* ctx, Round& rd) {
+  if (!rd.launched) return;
+  EIM_CUDA(cudaMemsetAsync(round_flags(rd) + 1, 0xFF, sizeof(unsigned int), ctx->aux_stream));
+}
+
+void round_resume(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st) {
+  if (!rd.launched) return;
+  EIM_CUDA(cudaStreamSynchronize(ctx->aux_stream));  // an earlier pause write lands before the clear below
+  EIM_CUDA(cudaStreamWaitEvent(st, rd.ev[2 * rd.nlaunch - 1], 0));
+  EIM_CUDA(cudaMemsetAsync(round_flags(rd) + 1, 0, sizeof(unsigned int), st));
+  round_kernel(ctx, g, rd, st, false);
 }
 
 void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first,
                   uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot) {
   if (count == 0) return;
-  if (count >= 0x7FFFFFF0ull) fail(EIM_E_INVAL, "at most 2^31 sets per sampler launch");
-  if (!rd.ev0) {
-    EIM_CUDA(cudaEventCreate(&rd.ev0));
-    EIM_CUDA(cudaEventCreate(&rd.ev1));
-  }
+  if (count >= 0x3FFFFFF0ull) fail(EIM_E_INVAL, "at most 2^30 sets per sampler launch");
+  if (!rd.ev[0])
+    for (cudaEvent_t& e : rd.ev) EIM_CUDA(cudaEventCreate(&e));
   rd.first = first;
   rd.count = count;
   rd.set_base = set_base;
@@ -554,7 +607,7 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   rd.failed.reserve(count, false, st);
   rd.edges.reserve(count * sizeof(unsigned long long), false, st);
   rd.fill.reserve(count * sizeof(uint32_t), false, st);
-  rd.retry.reserve(count * sizeof(uint32_t), false, st);
+  rd.retry.reserve(2 * count * sizeof(uint32_t), false, st);  // two retry lists (tier 1 -> 2 -> 3)
   rd.excl.reserve((count + 1) * sizeof(uint64_t), false, st);
   rd.ctl.reserve(sizeof(SampleCtl) + 16, false, st);
   // table capacity: >= 4x the expected members (mean set size of earlier
@@ -568,8 +621,7 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 
 void round_cancel(eim_ctx* ctx, Round& rd) {
   if (!rd.launched) return;
-  unsigned int* cancel = reinterpret_cast<unsigned int*>(rd.ctl.as<SampleCtl>() + 1);
-  EIM_CUDA(cudaMemsetAsync(cancel, 0xFF, sizeof(unsigned int), ctx->aux_stream));
+  EIM_CUDA(cudaMemsetAsync(round_flags(rd), 0xFF, sizeof(unsigned int), ctx->aux_stream));
   EIM_CUDA(cudaStreamSynchronize(ctx->aux_stream));
   EIM_CUDA(cudaStreamSynchronize(rd.stream));
   rd.launched = false;
@@ -582,37 +634,63 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   cudaStream_t st = ctx->stream;
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
   SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
+  auto elapsed = [&](int from) {
+    float total = 0, ms = 0;
+    for (int i = from; i < rd.nlaunch; ++i) {
+      EIM_CUDA(cudaEventElapsedTime(&ms, rd.ev[2 * i], rd.ev[2 * i + 1]));
+      total += ms;
+    }
+    return (double)total;
+  };
   for (int attempt = 0;; ++attempt) {
-    EIM_CUDA(cudaStreamWaitEvent(st, rd.ev1, 0));
-    EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
-    EIM_CUDA(cudaStreamSynchronize(st));
-    float ms = 0;
-    EIM_CUDA(cudaEventElapsedTime(&ms, rd.ev0, rd.ev1));
-    res.kernel_ms += ms;
-    res.launches++;
-    bool table_full = h->arena_fail != 0;
-    if (!table_full && h->retry_count > 0) {
-      // tier 2: a frontier backlog outgrew the shared ring; redo those samples
-      // with a 512-thread group and a global ring of capacity >= n
-      const uint64_t nretry = h->retry_count;
-      res.tier2 += nretry;
-      uint32_t W2 = 1;
-      while (W2 < g->view.n) W2 <<= 1;
-      uint64_t slots = std::min<uint64_t>(nretry, std::max<uint64_t>(1, (1ull << 30) / (4ull * W2)));
-      slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count);
-      ctx->tier_queue.reserve(slots * (uint64_t)W2 * 4, false, st);
-      EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
-      EIM_CUDA(cudaEventRecord(rd.ev0, st));
-      launch_ic<IC_G2, true>(ctx, g, rd.seed, round_view(rd), nretry, rd.retry.as<uint32_t>(), W2, ctl, nullptr,
-                             ctx->tier_queue.as<uint32_t>(), slots, st, false);
-      EIM_CUDA(cudaEventRecord(rd.ev1, st));
+    int counted = 0;
+    for (;;) {  // until the tier-1 launches have taken every id (a paused round is resumed here)
+      EIM_CUDA(cudaStreamWaitEvent(st, rd.ev[2 * rd.nlaunch - 1], 0));
       EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
       EIM_CUDA(cudaStreamSynchronize(st));
-      EIM_CUDA(cudaEventElapsedTime(&ms, rd.ev0, rd.ev1));
-      res.kernel_ms += ms;
-      res.launches++;
+      if (h->ticket >= rd.count || h->arena_fail) break;
+      round_resume(ctx, g, rd, st);
+    }
+    res.kernel_ms += elapsed(counted);
+    res.launches += rd.nlaunch - counted;
+    counted = rd.nlaunch;
+    bool table_full = h->arena_fail != 0;
+    // retry tiers over the ids a tier gave up: tier 2 = a whole SM (1024
+    // threads) per sample with a larger shared-memory ring (the long chains
+    // handed off by tier 1, and ring overflows); tier 3 = global-memory ring
+    // of capacity >= n, which cannot overflow
+    uint32_t* lists[2] = {rd.retry.as<uint32_t>(), rd.retry.as<uint32_t>() + rd.count};
+    if (!table_full && h->retry_count > 0)  // a pause that arrived after the last id was taken
+      EIM_CUDA(cudaMemsetAsync(round_flags(rd) + 1, 0, sizeof(unsigned int), st));
+    for (uint32_t tier = 1; !table_full && h->retry_count > 0; ++tier) {
+      if (tier > 2) fail(EIM_E_CUDA, "tier-3 sampler failed with a ring of capacity n");
+      const uint64_t nretry = h->retry_count;
+      res.tier2 += nretry;
+      uint32_t* in = lists[(tier - 1) & 1];
+      uint32_t* out = lists[tier & 1];
+      EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
+      if (rd.nlaunch >= Round::MAX_LAUNCH) fail(EIM_E_STATE, "too many sampler launches in one round");
+      EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch], st));
+      if (tier == 1) {
+        launch_ic<IC_G2, false>(ctx, g, rd.seed, round_view(rd), nretry, in, IC_W2, ctl, out, nullptr,
+                                ctx->sm_count, st, false, 1, 0);
+      } else {
+        uint32_t W3 = 1;
+        while (W3 < g->view.n) W3 <<= 1;
+        uint64_t slots = std::min<uint64_t>(nretry, std::max<uint64_t>(1, (1ull << 30) / (4ull * W3)));
+        slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count);
+        ctx->tier_queue.reserve(slots * (uint64_t)W3 * 4, false, st);
+        launch_ic<IC_G3, true>(ctx, g, rd.seed, round_view(rd), nretry, in, W3, ctl, out,
+                               ctx->tier_queue.as<uint32_t>(), slots, st, false, 2, 0);
+      }
+      EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch + 1], st));
+      rd.nlaunch++;
+      EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
+      EIM_CUDA(cudaStreamSynchronize(st));
+      res.kernel_ms += elapsed(counted);
+      res.launches += rd.nlaunch - counted;
+      counted = rd.nlaunch;
       table_full = h->arena_fail != 0;
-      if (!table_full && h->retry_count) fail(EIM_E_CUDA, "tier-2 sampler failed with a ring of capacity n");
     }
     if (table_full) {  // rare: redo the whole range with a 4x larger table
       if (attempt >= 4 || rd.bits >= 31) fail(EIM_E_NOMEM, "membership table overflow");

@@ -33,7 +33,7 @@ namespace eim {
 namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
-constexpr int GB = 256;  // threads per block of the greedy kernel (one block per SM: fits next to a running sampler)
+constexpr int GB = 512;  // threads per block of the greedy kernel
 
 __global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t* __restrict__ flags) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -258,9 +258,9 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   EIM_CUDA(cudaMemsetAsync(ctx->selected.p, 0, (uint64_t)n + 4, st));
   int per_sm = 0;
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
-  const char* gbe = getenv("EIM_GREEDY_BPSM");  // development: blocks per SM of the greedy kernel
-  const int bpsm = gbe ? atoi(gbe) : 1;
-  uint32_t blocks = (uint32_t)std::max(1, std::min(per_sm, bpsm)) * ctx->sm_count;
+  const char* gbe = getenv("EIM_GREEDY_BLOCKS");  // development: grid of the greedy kernel
+  uint32_t blocks = gbe ? (uint32_t)atoi(gbe) : (uint32_t)ctx->sm_count;
+  blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
   ctx->best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
   uint32_t* zc = reinterpret_cast<uint32_t*>(ctx->best.as<unsigned long long>() + blocks);
   EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
