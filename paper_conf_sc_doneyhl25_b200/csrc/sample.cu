@@ -128,6 +128,7 @@ struct RoundView {
   unsigned long long* edges;     // [count] examined in-edges (IC) / walk steps (LT) per sample
   const unsigned int* cancel;    // [0] cancel (round not needed), [1] pause (take no new ids)
   uint64_t base;                 // sample id of s_local = 0
+  PhiloxKey K;                   // round keys of the seed (kernel parameter: read as constant operands)
 };
 
 // One IC RRR set (Alg. 2 l.5-20) by a group of G threads.  ring = frontier
@@ -271,9 +272,15 @@ __device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const Ph
           Tk[k] = T_r;
         }
       }
+      // all U Philox calls before any branch (independent chains interleave);
+      // one 4-way min per quad against T decides whether the rare exact test runs
       uint4 wk[U];
 #pragma unroll
       for (int k = 0; k < U; ++k) wk[k] = philox_at(qk[k], s, TAG_EDGE, K);
+      bool any = false;
+#pragma unroll
+      for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
+      if (!any) continue;
 #pragma unroll
       for (int k = 0; k < U; ++k) {
         const uint32_t T = Tk[k];
@@ -332,7 +339,7 @@ __global__ void __launch_bounds__(G, (G >= 1024 ? 1 : (G >= 512 ? 2 : 6))) ic_gr
     rows_smem.T = reinterpret_cast<uint32_t*>(dyn + 16ull * W);
   }
   const RingRows* rr = GLOBAL_RING ? nullptr : &rows_smem;
-  const PhiloxKey K = philox_key(seed);
+  const PhiloxKey& K = R.K;
   unsigned long long edges_acc = 0;
   for (;;) {
     if (gtid == 0) {
@@ -536,7 +543,8 @@ static uint32_t handoff_threshold(eim_ctx*) {
 static RoundView round_view(Round& rd) {
   return RoundView{rd.table.as<unsigned long long>(), rd.bits, rd.sizes.as<uint32_t>(), rd.failed.as<uint8_t>(),
                    rd.edges.as<unsigned long long>(),
-                   reinterpret_cast<const unsigned int*>(rd.ctl.as<SampleCtl>() + 1), rd.first};
+                   reinterpret_cast<const unsigned int*>(rd.ctl.as<SampleCtl>() + 1), rd.first,
+                   philox_key(rd.seed)};
 }
 
 // one tier-1 sampler launch over rd's remaining ids, bracketed by events
