@@ -235,7 +235,7 @@ def main():
     theta_all = stats[-1]["theta"]
     value = theta_all / (ms_per_step / 1e3)
 
-    # dominant kernel: IC tier-1 sampler; per-launch duration from CUDA events on the ctx stream
+    # dominant kernel: IC sampler; per-launch duration from CUDA events on the ctx stream
     k_ms = sum(s["ms_sample_kernel"] for s in stats)
     k_launch = sum(s["sample_launches"] for s in stats)
     k_edges_local = sum(s["edges_examined"] for s in stats)
@@ -293,7 +293,7 @@ def main():
                          "sample_kernel": k_ms / args.steps,
                          "select": sum(s["ms_select"] for s in stats) / args.steps,
                          "comm": sum(s["ms_comm"] for s in stats) / args.steps},
-            "roofline": {"bound": "alu", "kernel": "ic_group_kernel (sampler, all tiers)", "achieved": achieved,
+            "roofline": {"bound": "alu", "kernel": "ic_kernel (IC sampler, incl. split-off tasks)", "achieved": achieved,
                          "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
                          "traffic": traffic,
                          "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge), "
@@ -305,7 +305,7 @@ def main():
             "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
             "clocks": clk,
             "result": {"seeds_head": seeds[:10].tolist(), "theta": theta_all, "spread": spread,
-                       "rounds": stats[-1]["rounds"], "tier2_samples": stats[-1]["tier2_samples"],
+                       "rounds": stats[-1]["rounds"], "spilled_samples": stats[-1]["spilled_samples"],
                        "edges_examined": stats[-1]["edges_examined"]},
         }
         print(json.dumps(out), flush=True)

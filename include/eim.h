@@ -59,14 +59,14 @@ typedef struct {
   uint64_t cov;                 /* coverage of the final seed set */
   uint64_t edges_examined;      /* IC: sum of d^-(u) over expanded u; LT: walk steps (local rank) */
   uint64_t arena_elems;         /* members stored in R (all ranks) */
-  uint64_t tier2_samples;       /* samples redone in a global-memory tier (local rank) */
+  uint64_t spilled_samples;     /* IC samples finished in the shared frontier queue (local rank) */
   uint64_t kernel_launches;     /* eim kernels launched by this call (local rank) */
-  uint32_t sample_launches;     /* tier-1 sampler launches */
+  uint32_t sample_launches;     /* sampler kernel launches */
   double ms_total;              /* wall time of the call (host clock) */
   double ms_sample;             /* wall time in sampling (incl. retries, exchange) */
   double ms_select;             /* wall time in greedy NodeSelection (incl. index build) */
   double ms_comm;               /* wall time in NCCL exchanges */
-  double ms_sample_kernel;      /* device time of the tier-1 sampler kernels (CUDA events on the ctx stream) */
+  double ms_sample_kernel;      /* device time of the sampler kernels (CUDA events on the ctx stream) */
 } eim_stats;
 
 /* IMM parameters of [22] (host-only, no device needed). */
@@ -160,7 +160,7 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
 
 /* Statistics of the most recent eim_imm_run / eim_sample_rrr call on ctx
  * (for eim_sample_rrr: theta = count, edges_examined, sample_launches,
- * tier2_samples, ms_sample_kernel, ms_sample, ms_total, arena_elems,
+ * spilled_samples, ms_sample_kernel, ms_sample, ms_total, arena_elems,
  * kernel_launches).  Errors: EIM_E_STATE, EIM_E_INVAL (out NULL). */
 eim_status eim_get_stats(const eim_ctx* ctx, eim_stats* out);
 

@@ -48,7 +48,7 @@ class Stats(ctypes.Structure):
         ("cov", ctypes.c_uint64),
         ("edges_examined", ctypes.c_uint64),
         ("arena_elems", ctypes.c_uint64),
-        ("tier2_samples", ctypes.c_uint64),
+        ("spilled_samples", ctypes.c_uint64),
         ("kernel_launches", ctypes.c_uint64),
         ("sample_launches", ctypes.c_uint32),
         ("ms_total", ctypes.c_double),

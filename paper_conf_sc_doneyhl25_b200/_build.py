@@ -35,8 +35,10 @@ def _nvcc():
 
 
 def _flags(extra_inc):
+    # EIM_NVCC_DEFS: extra -D flags for tuning experiments (build with --force)
+    defs = os.environ.get("EIM_NVCC_DEFS", "").split()
     return ["-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC,-ffp-contract=off,-fno-fast-math",
-            "-I", INCLUDE, "-I", CSRC, "-I", extra_inc, "--expt-relaxed-constexpr"]
+            "-I", INCLUDE, "-I", CSRC, "-I", extra_inc, "--expt-relaxed-constexpr", *defs]
 
 
 def build(force: bool = False, verbose: bool = False) -> str:

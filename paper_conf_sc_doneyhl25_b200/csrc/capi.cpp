@@ -88,8 +88,7 @@ eim_status guarded(eim_ctx* ctx, F&& f) {
 bool ctx_ok(const eim_ctx* ctx) { return ctx && ctx->magic == CTX_MAGIC; }
 
 void free_ctx_buffers(eim_ctx* c) {
-  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->retry_a, &c->retry_b,
-                    &c->tier_tab, &c->tier_queue, &c->tier_gen, &c->C_total, &c->C_work, &c->inv_off,
+  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->C_total, &c->C_work, &c->inv_off,
                     &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
                     &c->stage_b, &c->stage_c, &c->cand, &c->cidx, &c->arena_c, &c->selected};
   for (DevBuf* b : bufs) b->release();
@@ -268,7 +267,7 @@ eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
     const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false);
     std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
     ctx->last_stats.edges_examined = r.edges;
-    ctx->last_stats.tier2_samples = r.tier2;
+    ctx->last_stats.spilled_samples = r.spilled;
     ctx->last_stats.sample_launches = r.launches;
     ctx->last_stats.ms_sample_kernel = r.kernel_ms;
     ctx->last_stats.theta = count;

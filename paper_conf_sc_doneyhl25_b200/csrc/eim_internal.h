@@ -52,13 +52,19 @@ struct ArenaView {
 };
 
 // Per-launch control block (device memory).
+// Per-launch control block (device memory).  The counters that every group
+// polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
-  unsigned long long ticket;
-  unsigned long long retry_count;
-  unsigned long long edges;
-  unsigned long long arena_fail;
-  unsigned long long active;  // samples in progress (tier-1 tail hand-off)
-  unsigned long long pad;
+  unsigned long long ticket, pad0[15];          // next sample id (s_local)
+  unsigned long long thead, ttail, pad1[14];    // task descriptors: next to take, reserved
+  unsigned long long ptail, pad2[15];           // task seed pool: reserved
+  unsigned long long outstanding, pad3[15];     // samples + tasks taken or queued, not finished
+  unsigned long long edges;                     // examined in-edges / walk steps (finalize)
+  unsigned long long arena_fail;                // table or task pool full: redo the round larger
+  unsigned long long spilled;                   // samples that split off tasks
+  unsigned long long tasks_pushed;              // tasks split off
+  unsigned long long t_first, t_last_id, t_end;  // %globaltimer: first id taken, last id taken, last group exit (timeline)
+  unsigned long long pad4[9];
 };
 
 struct Comm;  // NCCL communicator wrapper (comm.cpp)
@@ -67,8 +73,11 @@ struct Comm;  // NCCL communicator wrapper (comm.cpp)
 // table and per-sample scratch.  Two of them let the IMM driver sample the
 // next round speculatively while the greedy of the current round runs.
 struct Round {
-  DevBuf table, sizes, failed, edges, fill, retry, excl, ctl;  // ctl: SampleCtl + cancel flag
-  uint64_t first = 0, count = 0, set_base = 0, seed = 0;
+  DevBuf table, sizes, edges, fill, excl, ctl;  // ctl: SampleCtl + cancel/pause flags
+  DevBuf dbg;                                    // EIM_DEBUG_TIMELINE per-sample records
+  DevBuf queue;                                  // IC task pool (u32 seeds) + descriptors (all-zero between rounds)
+  uint64_t first = 0, count = 0, set_base = 0, seed = 0, pcap = 0, tcap = 0;
+  bool qdirty = true;                            // descriptors need a memset before use
   uint32_t bits = 0;
   eim_model model = EIM_IC;
   cudaStream_t stream = nullptr;  // stream the sampler kernels were launched on
@@ -103,8 +112,6 @@ struct eim_ctx {
   // arena (persistent, grows)
   eim::DevBuf arena, set_start, set_len, covered;
   eim::DevBuf ctl;            // SampleCtl
-  eim::DevBuf retry_a, retry_b;
-  eim::DevBuf tier_tab, tier_queue, tier_gen;  // global-memory tiers
   eim::Round rounds[2];                         // current + speculative sampler rounds
   cudaStream_t rstream[2] = {};                 // sampler streams of rounds[0], rounds[1]
   cudaStream_t aux_stream = nullptr;            // cancel-flag writes
@@ -132,7 +139,7 @@ void graph_validate_and_thresholds(eim_ctx* ctx, eim_graph* g);
 // ---- sample.cu
 struct SampleResult {
   uint64_t edges = 0;
-  uint64_t tier2 = 0;
+  uint64_t spilled = 0;   // samples finished in the shared frontier queue
   uint32_t launches = 0;
   double kernel_ms = 0;
 };

@@ -55,7 +55,7 @@ void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   eim_shard_range(R, R_new - R, ctx->rank, ctx->world, &lo, &hi);
   SampleResult r = sample_range(ctx, g, model, seed, lo, hi - lo, 0, false);
   st->edges_examined += r.edges;
-  st->tier2_samples += r.tier2;
+  st->spilled_samples += r.spilled;
   st->sample_launches += r.launches;
   st->ms_sample_kernel += r.kernel_ms;
   const auto tc = clk::now();
@@ -172,7 +172,7 @@ class RoundSampler {
   cudaStream_t stream_of(const Round& rd) const { return &rd == &ctx_->rounds[0] ? ctx_->rstream[0] : ctx_->rstream[1]; }
   void account(const SampleResult& r) {
     st_->edges_examined += r.edges;
-    st_->tier2_samples += r.tier2;
+    st_->spilled_samples += r.spilled;
     st_->sample_launches += r.launches;
     st_->ms_sample_kernel += r.kernel_ms;
   }

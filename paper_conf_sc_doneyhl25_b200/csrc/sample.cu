@@ -10,22 +10,27 @@
 // every member into the arena and bumps the coverage histogram C (Alg. 2 l.25)
 // -- placement is deterministic, no reservation atomics, no arena overflow.
 //
-// IC (ic_group_kernel<G, GLOBAL_RING>): G threads cooperate on one sample.  A
-//   batch of up to G frontier vertices has its in-rows merged into one space
-//   of Philox quads (4 consecutive edge ids share one Philox4x32-10 call,
-//   reading R1) that the G threads sweep, so small rows do not idle threads
-//   and hub rows split evenly.  An edge into u is live iff its draw <= T_u
-//   (R2); in_nbr[e] is read only for live edges.  Heavy samples under WC are
-//   chains of ~100 hub expansions, so G threads per sample (not a warp) keep
-//   the per-level latency low, and they start as soon as their id is drawn.
-//   The frontier lives in a shared-memory ring (tier 1); a sample whose
-//   backlog outgrows the ring is redone by a 512-thread group with the ring
-//   in global memory (tier 2, capacity n) under a distinct key tag.
+// IC (ic_kernel<G>): persistent groups of G threads.  A group takes a sample
+//   id and runs it in shared memory (local_sample): a batch of up to G
+//   frontier vertices has its in-rows merged into one space of Philox quads
+//   (4 consecutive edge ids share one Philox4x32-10 call, reading R1) that
+//   the G threads sweep, so small rows do not idle threads and hub rows split
+//   evenly.  An edge into u is live iff its draw <= T_u (R2); in_nbr[e] is
+//   read only for live edges.  Under WC a few samples per round are huge
+//   (~10^5 members, ~10^6 quads): on one group they would bound the round.
+//   So after every spill_quads swept quads a traversal cuts its backlog into
+//   pieces of about task_quads quads each, keeps one and pushes the others as
+//   TASKS (a sample id and its seed vertices) that any group runs the same
+//   way, before it takes a new id.  Membership stays in the round table (first insert wins
+//   and expands the vertex), so nothing is redone and the union of the
+//   traversals is the unique reachable set.
 // LT (lt_kernel): one thread per reverse walk (sequential by nature),
 //   visited set = the same global table; no capacity limit.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <cstdio>
+#include <vector>
 #include <cstdlib>
 #include <string>
 
@@ -39,16 +44,24 @@ namespace {
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr uint32_t MAX_PROBE = 256;
 
-constexpr int IC_G = 256;          // threads per sample (one block), tier 1
-constexpr int IC_NG = 1;           // groups per block
-constexpr int IC_U = 2;            // consecutive quads per thread per sweep iteration
+#ifndef EIM_IC_G
+#define EIM_IC_G 256
+#endif
+#ifndef EIM_IC_NSG
+#define EIM_IC_NSG 1
+#endif
+constexpr int IC_G = EIM_IC_G;      // threads per sub-group (one traversal at a time)
+constexpr int IC_NSG = EIM_IC_NSG;  // sub-groups per block (one block per SM)
+constexpr int U_IC = 2;             // quads per lane per sweep step (independent Philox chains)
+#ifndef EIM_PARK_EDGE
+#define EIM_PARK_EDGE 1  // 1: park live edge ids and load their in-neighbours in the visit phase
+#endif
 
 // ---------------------------------------------------------------- table
-// key = ((s_local + 1) | tier << 30) << 32 | v ;  0 = empty slot.  tier =
-// attempt number of the sample (0, 1, 2): the scatter keeps only the keys of
-// the attempt that succeeded.
-__device__ __forceinline__ unsigned long long table_key(uint32_t s_local, uint32_t tier, uint32_t v) {
-  return ((unsigned long long)((s_local + 1u) | (tier << 30)) << 32) | (unsigned long long)v;
+// key = (s_local + 1) << 32 | v ;  0 = empty slot.  The same 64-bit word is
+// the item format of the shared frontier queue.
+__device__ __forceinline__ unsigned long long table_key(uint32_t s_local, uint32_t v) {
+  return ((unsigned long long)(s_local + 1u) << 32) | (unsigned long long)v;
 }
 
 __device__ __forceinline__ uint32_t table_hash(unsigned long long key, uint32_t bits) {
@@ -71,15 +84,41 @@ __device__ __forceinline__ int table_insert(unsigned long long* keys, uint32_t b
   return -1;
 }
 
-// ---------------------------------------------------------------- groups
-// One group = one block (G = blockDim.x), so a group barrier is __syncthreads.
-template <int G>
-__device__ __forceinline__ void gsync(int) {
-  __syncthreads();
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
 }
+
+__device__ __forceinline__ unsigned long long vload(const unsigned long long* p) {
+  return *(const volatile unsigned long long*)p;
+}
+
+// ---------------------------------------------------------------- groups
+// A block is NSG sub-groups of G threads.  A sub-group runs one traversal at
+// a time and synchronises on its own named barrier; the sub-groups of a
+// block share nothing but the sweep jobs below (shared memory).
+template <int G>
+__device__ __forceinline__ void gsync(int gi) {
+  asm volatile("bar.sync %0, %1;" ::"r"(gi + 1), "r"(G) : "memory");
+}
+
+// Sweep job of a sub-group's current batch.  Warps claim chunks of ch quads
+// through `claim` = epoch << 48 | nchunks << 24 | next chunk (an old epoch or
+// next >= nchunks claims nothing), so the warps of the other sub-groups of
+// the block can join a heavy batch (open = 1) between their own batches or
+// when they are idle.  done counts finished chunks of the epoch.
+struct Job {
+  unsigned long long claim;
+  uint32_t done, open;
+  uint32_t total, nrows, s_local, head, ch, pad;
+};
 
 struct GroupCtl {
   uint32_t tail, flag, s_local, nlive;
+  uint32_t pushed, action, nb, epoch;  // pushed: this traversal split off a task
+  unsigned long long h, base;
+  Job job;
   uint32_t wsum[32];  // one per warp (G <= 1024)
 };
 
@@ -100,288 +139,706 @@ __device__ __forceinline__ uint32_t group_incl_scan(uint32_t x, int gtid, int gi
     const uint32_t t = __shfl_up_sync(FULL, x, o);
     if (lane >= o) x += t;
   }
-  if constexpr (G == 32) {
-    total = __shfl_sync(FULL, x, 31);
-    return x;
-  } else {
-    if (lane == 31) gc.wsum[w] = x;
-    gsync<G>(gi);
-    uint32_t pre = 0, tot = 0;
+  if (lane == 31) gc.wsum[w] = x;
+  gsync<G>(gi);
+  uint32_t pre = 0, tot = 0;
 #pragma unroll
-    for (int i = 0; i < G / 32; ++i) {
-      const uint32_t t = gc.wsum[i];
-      pre += (i < w) ? t : 0u;
-      tot += t;
-    }
-    total = tot;
-    return x + pre;
+  for (int i = 0; i < G / 32; ++i) {
+    const uint32_t t = gc.wsum[i];
+    pre += (i < w) ? t : 0u;
+    tot += t;
   }
+  total = tot;
+  return x + pre;
 }
 
-enum : uint32_t { FLAG_RING = 1u, FLAG_TABLE = 2u, FLAG_CANCEL = 4u, FLAG_HANDOFF = 8u };
+enum : uint32_t { FLAG_TABLE = 2u, FLAG_CANCEL = 4u };
+enum : uint32_t { ACT_EXIT = 0u, ACT_LOCAL = 1u, ACT_TASK = 2u, ACT_IDLE = 3u };
 
 struct RoundView {
   unsigned long long* keys;
   uint32_t bits;
   uint32_t* sizes;               // [count] members per sample (s_local)
-  uint8_t* failed;               // [count] attempt (tier) whose keys are the sample's members
-  unsigned long long* edges;     // [count] examined in-edges (IC) / walk steps (LT) per sample
-  const unsigned int* cancel;    // [0] cancel (round not needed), [1] pause (take no new ids)
+  unsigned long long* edges;     // [count] walk steps per sample (LT)
+  const unsigned int* cancel;    // [0] cancel (round not needed), [1] pause (take no new work)
   uint64_t base;                 // sample id of s_local = 0
+  uint32_t* pool;                // task seed vertices
+  unsigned long long* tasks;     // task descriptors: [2i] pool offset, [2i+1] (s_local+1) << 32 | nv (0 = unwritten)
+  uint64_t pcap, tcap;           // pool / descriptor capacity
+  unsigned long long* dbg;       // [count][8] per root traversal (EIM_DEBUG_TIMELINE), nullable
   PhiloxKey K;                   // round keys of the seed (kernel parameter: read as constant operands)
 };
 
-// One IC RRR set (Alg. 2 l.5-20) by a group of G threads.  ring = frontier
-// backlog of capacity W (W a power of two).  Returns the flag (0 = success);
-// size = number of members.
+constexpr uint32_t LIVE_CAP = 512;  // live in-edges parked per batch (more are visited inline)
+
 // Row descriptors of queued frontier vertices, loaded when the vertex is
-// discovered (tier 1): the next batch stages its rows from shared memory.
+// discovered: the next batch stages its rows from shared memory.
 struct RingRows {
   unsigned long long* e0;  // [W] first in-edge
   uint32_t* d;             // [W] in-degree
   uint32_t* T;             // [W] IC threshold
 };
 
-constexpr uint32_t LIVE_CAP = 512;  // live in-edges buffered per batch (more are visited inline)
+// One sub-group's shared-memory region.
+template <int G>
+struct SG {
+  GroupCtl* gc;
+  GroupRows<G>* rw;
+  RingRows rr;
+  uint32_t* ring;
+  unsigned long long* live_e;  // parked live edges of the current batch
+};
 
-// One IC RRR set (Alg. 2 l.5-20) by a group of G threads.  ring = frontier
-// backlog of capacity W (W a power of two); rr (nullable) = prefetched rows
-// of the ring entries.  A batch is three phases separated by group
-// barriers: stage up to G queued rows and scan their Philox-quad counts;
-// sweep the quads (Philox + compare only; the in-neighbour of a live edge is
-// loaded and parked in a shared list); visit the parked neighbours in
-// parallel (one table insert each; a new member joins the ring with its row
-// bounds).  Separating the visits keeps the long-latency loads and atomics of
-// the rare live edges off the Philox sweep and runs them side by side, which
-// bounds the per-level latency of long chains.  Returns the flag (0 = ok).
+template <int G>
+__host__ __device__ constexpr size_t sg_bytes(uint32_t W) {
+  return (sizeof(GroupCtl) + sizeof(GroupRows<G>) + 20ull * W + 8ull * LIVE_CAP + 15) & ~(size_t)15;
+}
+
+template <int G>
+__device__ __forceinline__ SG<G> sg_at(unsigned char* smem, int gi, uint32_t W) {
+  unsigned char* p = smem + (size_t)gi * sg_bytes<G>(W);
+  SG<G> r;
+  r.gc = reinterpret_cast<GroupCtl*>(p);
+  p += sizeof(GroupCtl);
+  r.rw = reinterpret_cast<GroupRows<G>*>(p);
+  p += sizeof(GroupRows<G>);
+  r.rr.e0 = reinterpret_cast<unsigned long long*>(p);
+  p += 8ull * W;
+  r.ring = reinterpret_cast<uint32_t*>(p);
+  p += 4ull * W;
+  r.rr.d = reinterpret_cast<uint32_t*>(p);
+  p += 4ull * W;
+  r.rr.T = reinterpret_cast<uint32_t*>(p);
+  p += 4ull * W;
+  r.live_e = reinterpret_cast<unsigned long long*>(p);
+  return r;
+}
+
+__device__ __forceinline__ void mark_fail(SampleCtl* ctl) {
+  atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);
+}
+
+// Publish task i: descriptor word 0 (pool offset) is made visible before
+// word 1, which a consumer spins on.
+__device__ __forceinline__ void task_write(const RoundView& R, unsigned long long i, unsigned long long poff,
+                                           uint32_t s_local, uint32_t nv) {
+  R.tasks[2 * i] = poff;
+  __threadfence();
+  *(volatile unsigned long long*)&R.tasks[2 * i + 1] = ((unsigned long long)(s_local + 1u) << 32) | nv;
+}
+
+// Push one vertex as a task of its own (ring overflow; rare).  outstanding is
+// raised before the task becomes visible.
+__device__ __forceinline__ void task_push1(const RoundView& R, SampleCtl* ctl, uint32_t s_local, uint32_t v) {
+  atomicAdd(&ctl->outstanding, 1ull);
+  const unsigned long long po = atomicAdd(&ctl->ptail, 1ull);
+  const unsigned long long ti = atomicAdd(&ctl->ttail, 1ull);
+  if (ti >= R.tcap) {  // descriptor array full: host redoes the round larger
+    mark_fail(ctl);
+    atomicAdd(&ctl->outstanding, ~0ull);
+    return;
+  }
+  if (po >= R.pcap) {  // pool full: an empty task keeps the claimed slot consumable
+    mark_fail(ctl);
+    task_write(R, ti, 0, s_local, 0);
+    return;
+  }
+  R.pool[po] = v;
+  __threadfence();
+  task_write(R, ti, po, s_local, 1);
+}
+
+// visit v for the traversal of sub-group o (sample s_local, ring head `head`):
+// table insert; a new member is appended to o's ring with its row (loaded
+// alongside the insert), or becomes a one-vertex task when the ring is full.
+template <int G>
+__device__ __forceinline__ void visit_for(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                          uint32_t s_local, uint32_t head, uint32_t W, uint32_t v) {
+  const unsigned long long e0 = g.off[v], e1 = g.off[v + 1];
+  const uint32_t T = g.thr[v];
+  const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
+  if (ins > 0) {
+    const uint32_t pos = atomicAdd(&o.gc->tail, 1u);
+    if (pos - head < W) {
+      const uint32_t sl = pos & (W - 1);
+      o.ring[sl] = v;
+      o.rr.e0[sl] = e0;
+      o.rr.d[sl] = (uint32_t)(e1 - e0);
+      o.rr.T[sl] = T;
+    } else {
+      task_push1(R, ctl, s_local, v);
+      o.gc->pushed = 1u;
+    }
+  } else if (ins < 0) {
+    atomicOr(&o.gc->flag, FLAG_TABLE);
+  }
+}
+
+// Light batch: the sub-group's G threads sweep all quads of its staged batch,
+// thread t taking quads t, t + G, .. in groups of U independent Philox chains
+// (rows found by an incremental walk over the scan).
 template <int G, int U>
-__device__ __forceinline__ uint32_t ic_group_sample(const GraphView& g, const PhiloxKey& K, const RoundView& R,
-                                                    uint32_t s_local, uint32_t tier, uint32_t* ring, uint32_t W,
-                                                    const RingRows* rr, uint32_t* live_v, GroupRows<G>& rw,
-                                                    GroupCtl& gc, int gtid, int gi, unsigned long long& se,
-                                                    uint32_t& size, const SampleCtl* ctl, uint64_t count,
-                                                    uint32_t handoff) {
-  const uint64_t s = R.base + s_local;
-  uint32_t head = 0;
-  // visit v: table insert; a new member is appended to the ring (with its row)
-  auto visit = [&](uint32_t v) {
-    const int ins = table_insert(R.keys, R.bits, table_key(s_local, tier, v));
-    if (ins > 0) {
-      const uint32_t pos = atomicAdd(&gc.tail, 1u);
-      if (pos - head < W) {
-        const uint32_t sl = pos & (W - 1);
-        ring[sl] = v;
-        if (rr) {
-          const unsigned long long e0 = g.off[v];
-          rr->e0[sl] = e0;
-          rr->d[sl] = (uint32_t)(g.off[v + 1] - e0);
-          rr->T[sl] = g.thr[v];
+__device__ __forceinline__ void sweep_strided(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                              uint32_t total, int gtid, uint32_t c2, uint32_t c3, uint32_t s_local,
+                                              uint32_t head, uint32_t W) {
+  const GroupRows<G>& rw = *o.rw;
+  int r = -1;
+  uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0;
+  unsigned long long q0_r = 0;
+  for (uint32_t base = 0; base < total; base += U * G) {
+    unsigned long long qk[U];
+    uint32_t Tk[U], mk[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      const uint32_t j = base + k * G + gtid;
+      mk[k] = 0u;
+      qk[k] = 0ull;
+      Tk[k] = 0u;
+      if (j < total) {
+        if (j >= qe) {
+          do {
+            ++r;
+            qe = rw.qend[r];
+          } while (j >= qe);
+          nq_r = rw.nq[r];
+          qb = qe - nq_r;
+          q0_r = rw.q0[r];
+          T_r = rw.T[r];
+          wlo_r = rw.wlo[r];
+          whi_r = rw.whi[r];
         }
-      } else {
-        atomicOr(&gc.flag, FLAG_RING);
+        const uint32_t li = j - qb;
+        uint32_t m = 0xFu;
+        if (li == 0) m &= 0xFu << wlo_r;
+        if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
+        mk[k] = m;
+        qk[k] = q0_r + li;
+        Tk[k] = T_r;
       }
-    } else if (ins < 0) {
-      atomicOr(&gc.flag, FLAG_TABLE);
+    }
+    uint4 wk[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) wk[k] = philox((uint32_t)qk[k], (uint32_t)(qk[k] >> 32), c2, c3, R.K);
+    bool any = false;
+#pragma unroll
+    for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
+    if (!any) continue;
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      const uint32_t T = Tk[k];
+      uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
+                      (wk[k].w <= T ? 8u : 0u);
+      live &= mk[k];
+      while (live) {
+        const int i = __ffs(live) - 1;
+        live &= live - 1;
+        const unsigned long long e = (qk[k] << 2) + i;
+#if EIM_PARK_EDGE
+        // park the edge, not its in-neighbour: the visit phase loads them side by side
+        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
+        if (p < LIVE_CAP) o.live_e[p] = e;
+        else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
+#else
+        const uint32_t v = g.nbr[e];
+        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
+        if (p < LIVE_CAP) o.live_e[p] = v;
+        else visit_for<G>(g, R, ctl, o, s_local, head, W, v);
+#endif
+      }
+    }
+  }
+}
+
+// One warp sweeps quads [lo, hi) of o's staged batch (nrows rows; sample
+// counter words c2, c3): lane l takes quads lo + l, lo + l + 32, .. in
+// groups of U independent Philox chains; an edge into the row's vertex is
+// live iff its draw <= T (R2); the in-neighbour of a live edge is parked in
+// o's live list (visited directly when the list is full).
+template <int G, int U>
+__device__ __forceinline__ void sweep_chunk(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                            uint32_t nrows, uint32_t lo, uint32_t hi, int lane, uint32_t c2,
+                                            uint32_t c3, uint32_t s_local, uint32_t head, uint32_t W) {
+  const GroupRows<G>& rw = *o.rw;
+  // row of the chunk's first quad lo: first r with qend[r] > lo, found by
+  // the warp in two ballots over <= 32 x 8 rows (the lanes then walk on)
+  int r = 0;
+  {
+    const int seg = ((int)nrows + 31) >> 5;  // rows per lane segment (<= 8 for G = 256)
+    const int last = min((lane + 1) * seg, (int)nrows) - 1;
+    const bool past = last >= 0 && last >= lane * seg && rw.qend[last] > lo;
+    const unsigned bal = __ballot_sync(FULL, past);
+    const int L = bal ? __ffs(bal) - 1 : 31;
+    const int r0 = L * seg;
+    const int idx = r0 + lane;
+    const bool p2 = lane < seg && idx < (int)nrows && rw.qend[idx] > lo;
+    const unsigned b2 = __ballot_sync(FULL, p2);
+    r = b2 ? r0 + __ffs(b2) - 1 : (int)nrows - 1;
+  }
+  uint32_t qe = rw.qend[r], nq_r = rw.nq[r], qb = qe - nq_r, T_r = rw.T[r], wlo_r = rw.wlo[r], whi_r = rw.whi[r];
+  unsigned long long q0_r = rw.q0[r];
+  for (uint32_t base = lo; base < hi; base += 32 * U) {
+    unsigned long long qk[U];
+    uint32_t Tk[U], mk[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      const uint32_t j = base + k * 32 + lane;
+      mk[k] = 0u;
+      qk[k] = 0ull;
+      Tk[k] = 0u;
+      if (j < hi) {
+        if (j >= qe) {
+          do {
+            ++r;
+            qe = rw.qend[r];
+          } while (j >= qe);
+          nq_r = rw.nq[r];
+          qb = qe - nq_r;
+          q0_r = rw.q0[r];
+          T_r = rw.T[r];
+          wlo_r = rw.wlo[r];
+          whi_r = rw.whi[r];
+        }
+        const uint32_t li = j - qb;
+        uint32_t m = 0xFu;
+        if (li == 0) m &= 0xFu << wlo_r;
+        if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
+        mk[k] = m;
+        qk[k] = q0_r + li;
+        Tk[k] = T_r;
+      }
+    }
+    // all U Philox calls before any branch (independent chains interleave);
+    // one 4-way min per quad against T decides whether the rare exact test runs
+    uint4 wk[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) wk[k] = philox((uint32_t)qk[k], (uint32_t)(qk[k] >> 32), c2, c3, R.K);
+    bool any = false;
+#pragma unroll
+    for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
+    if (!any) continue;
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      const uint32_t T = Tk[k];
+      uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
+                      (wk[k].w <= T ? 8u : 0u);
+      live &= mk[k];
+      while (live) {
+        const int i = __ffs(live) - 1;
+        live &= live - 1;
+        const unsigned long long e = (qk[k] << 2) + i;
+#if EIM_PARK_EDGE
+        // park the edge, not its in-neighbour: the visit phase loads them side by side
+        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
+        if (p < LIVE_CAP) o.live_e[p] = e;
+        else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
+#else
+        const uint32_t v = g.nbr[e];
+        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
+        if (p < LIVE_CAP) o.live_e[p] = v;
+        else visit_for<G>(g, R, ctl, o, s_local, head, W, v);
+#endif
+      }
+    }
+  }
+}
+
+// A warp claims and sweeps chunks of o's current job until none is left.
+// Returns true if it swept anything.
+template <int G, int U>
+__device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                         int lane, uint32_t W) {
+  Job& j = o.gc->job;
+  bool any = false;
+  for (;;) {
+    unsigned long long old = 0;
+    if (lane == 0) {
+      old = *(volatile unsigned long long*)&j.claim;
+      if ((old & 0xFFFFFFull) < ((old >> 24) & 0xFFFFFFull)) old = atomicAdd(&j.claim, 1ull);
+    }
+    old = __shfl_sync(FULL, old, 0);
+    const uint32_t c = (uint32_t)(old & 0xFFFFFFull), n = (uint32_t)((old >> 24) & 0xFFFFFFull);
+    if (c >= n) return any;
+    // the job's fields are stable until this chunk is counted done
+    const uint32_t ch = *(volatile uint32_t*)&j.ch, total = *(volatile uint32_t*)&j.total;
+    const uint32_t nrows = *(volatile uint32_t*)&j.nrows, s_local = *(volatile uint32_t*)&j.s_local;
+    const uint32_t head = *(volatile uint32_t*)&j.head;
+    const uint64_t s = R.base + s_local;
+    const uint32_t lo = c * ch, hi = min(lo + ch, total);
+    sweep_chunk<G, U>(g, R, ctl, o, nrows, lo, hi, lane, (uint32_t)s, ctr_hi(s, TAG_EDGE), s_local, head, W);
+    __syncwarp();
+    __threadfence_block();  // parks and ring writes before the chunk counts as done
+    if (lane == 0) atomicAdd(&j.done, 1u);
+    any = true;
+  }
+}
+
+// Warp-level: join the open jobs of the other sub-groups of the block.
+template <int G, int NSG, int U>
+__device__ __forceinline__ bool help_others(const GraphView& g, const RoundView& R, SampleCtl* ctl,
+                                            unsigned char* smem, int gi, int lane, uint32_t W) {
+  bool any = false;
+  if (NSG < 2) return false;
+#pragma unroll 1
+  for (int k = 1; k < NSG; ++k) {
+    const int o = (gi + k) % NSG;
+    const SG<G> so = sg_at<G>(smem, o, W);
+    if (!*(volatile uint32_t*)&so.gc->job.open) continue;
+    any |= work_job<G, U>(g, R, ctl, so, lane, W);
+  }
+  return any;
+}
+
+// Stage one row (in-edges [e0, e1), threshold T) into slot gtid of rw;
+// returns its quad count.
+template <int G>
+__device__ __forceinline__ uint32_t stage_row(GroupRows<G>& rw, int gtid, unsigned long long e0,
+                                              unsigned long long e1, uint32_t T) {
+  uint32_t nq = 0;
+  if (e1 > e0) {
+    nq = (uint32_t)(((e1 - 1) >> 2) - (e0 >> 2) + 1);
+    rw.q0[gtid] = e0 >> 2;
+    rw.wlo[gtid] = (uint8_t)(e0 & 3);
+    rw.whi[gtid] = (uint8_t)((e1 - 1) & 3);
+    rw.T[gtid] = T;
+  }
+  rw.nq[gtid] = nq;
+  return nq;
+}
+
+// One traversal of sample s_local (Alg. 2 l.5-20) by sub-group gi in shared
+// memory: from the root, or from the nseed vertices of a task at pool[poff..]
+// (already members).  The ring is the frontier backlog of capacity W (a
+// power of two) with prefetched rows.  A batch: (1) stage up to G queued
+// rows and scan their Philox-quad counts; (2) sweep the quads as a job whose
+// chunks the sub-group's warps -- and, for a heavy batch, the idle warps of
+// the block's other sub-groups -- claim; (3) visit the parked live neighbours
+// in parallel (one table insert each; a new member joins the ring with its
+// row).  Between batches the sub-group helps the open jobs of its block.
+// After every spill_quads swept quads the backlog is cut into pieces of
+// about task_quads quads (heavy samples are chains of hub rows: few
+// vertices, many quads); one piece stays, the others become tasks that any
+// sub-group of the launch runs the same way.  Membership lives in the round
+// table (first insert wins, the winner expands the vertex), so the union of
+// the traversals is the unique reachable set of the sampled world, whatever
+// the split.  Returns 0, FLAG_TABLE or FLAG_CANCEL; found = new members
+// inserted by this traversal.
+template <int G, int NSG, int U>
+__device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView& R, SampleCtl* ctl,
+                                             unsigned char* smem, int gi, uint32_t s_local, bool root,
+                                             unsigned long long poff, uint32_t nseed, uint32_t W, int gtid,
+                                             uint32_t& found, uint32_t spill_quads, uint32_t task_quads,
+                                             uint32_t help_min, bool& split_any) {
+  const SG<G> me = sg_at<G>(smem, gi, W);
+  GroupCtl& gc = *me.gc;
+  GroupRows<G>& rw = *me.rw;
+  const int lane = gtid & 31;
+  const uint64_t s = R.base + s_local;
+  uint32_t head = 0, extra = 0;  // extra: members found here that left the ring (split off / overflow)
+  uint32_t swept = 0;
+  unsigned long long nbatch = 0, nquads = 0, t0 = (R.dbg && root && gtid == 0) ? gtimer() : 0ull;
+  unsigned long long ph[3] = {0, 0, 0}, tp = 0, nlive_tot = 0;  // ns in stage+scan, sweep, visit
+  auto dbg_end = [&]() {
+    if (R.dbg && root && gtid == 0) {
+      unsigned long long* d = R.dbg + 8ull * s_local;
+      d[0] = nbatch;
+      d[1] = nquads;
+      d[2] = t0;
+      d[3] = gtimer();
+      d[4] = ph[0];
+      d[5] = ph[1];
+      d[6] = ph[2];
+      d[7] = nlive_tot;
+    }
+  };
+  auto mark = [&](int i) {
+    if (R.dbg && gtid == 0) {
+      const unsigned long long t = gtimer();
+      if (i >= 0) ph[i] += t - tp;
+      tp = t;
     }
   };
   if (gtid == 0) {
-    gc.tail = 0;
     gc.flag = 0;
     gc.nlive = 0;
-    visit(draw_root(s, g.n, K));
+    gc.pushed = 0;
+    gc.tail = nseed;
+  }
+  if (root) {
+    gsync<G>(gi);
+    if (gtid == 0) visit_for<G>(g, R, ctl, me, s_local, 0, W, draw_root(s, g.n, R.K));
+  } else {
+    // pool lines may be cached from a neighbouring task: read through L2
+    for (uint32_t t = gtid; t < nseed; t += G) {
+      const uint32_t v = __ldcg(R.pool + poff + t);
+      const unsigned long long e0 = g.off[v];
+      me.ring[t] = v;
+      me.rr.e0[t] = e0;
+      me.rr.d[t] = (uint32_t)(g.off[v + 1] - e0);
+      me.rr.T[t] = g.thr[v];
+    }
   }
   gsync<G>(gi);
-  se = 0;
   for (;;) {
-    const uint32_t tail = *(volatile uint32_t*)&gc.tail;
+    uint32_t tail = *(volatile uint32_t*)&gc.tail;
     const uint32_t flag = *(volatile uint32_t*)&gc.flag;
-    if (flag || head >= tail) {
-      size = tail;
+    if (flag) {
+      found = tail + extra - nseed;
+      split_any = gc.pushed || extra;
       return flag;
+    }
+    if (tail - head > W) {  // positions past head + W went out as one-vertex tasks
+      extra += tail - head - W;
+      tail = head + W;
+    }
+    uint32_t npieces = 1;
+    if (spill_quads && swept >= spill_quads && tail - head >= 2) {
+      // quads of the backlog (rows are in rr) -> number of pieces
+      const uint32_t B = tail - head;
+      uint32_t q = 0;
+      for (uint32_t i = gtid; i < B; i += G) q += (me.rr.d[(head + i) & (W - 1)] + 3u) >> 2;
+      for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(FULL, q, o);
+      gsync<G>(gi);  // every thread has read gc.tail; wsum is free
+      if (lane == 0) gc.wsum[gtid >> 5] = q;
+      gsync<G>(gi);
+      uint32_t qb = 0;
+#pragma unroll
+      for (int i = 0; i < G / 32; ++i) qb += gc.wsum[i];
+      npieces = min(B, qb / max(task_quads, 1u));
+      if (npieces < 2) swept = spill_quads / 2;  // look again after a few batches
+    }
+    if (npieces >= 2) {
+      // ---- split: keep the first piece of tv vertices, push the rest as tasks of <= tv
+      const uint32_t B = tail - head;
+      const uint32_t tv = (B + npieces - 1) / npieces;
+      const uint32_t npush = B - tv;
+      const uint32_t ntasks = (npush + tv - 1) / tv;
+      gsync<G>(gi);  // every thread has read wsum
+      if (gtid == 0) {
+        atomicAdd(&ctl->outstanding, (unsigned long long)ntasks);
+        gc.base = atomicAdd(&ctl->ptail, (unsigned long long)npush);
+        gc.h = atomicAdd(&ctl->ttail, (unsigned long long)ntasks);
+        atomicAdd(&ctl->tasks_pushed, (unsigned long long)ntasks);
+      }
+      gsync<G>(gi);
+      const unsigned long long po = gc.base, ti = gc.h;
+      const bool ok = po + npush <= R.pcap;
+      if (ok)
+        for (uint32_t i = gtid; i < npush; i += G) R.pool[po + i] = me.ring[(head + tv + i) & (W - 1)];
+      __threadfence();
+      gsync<G>(gi);
+      for (uint32_t t = gtid; t < ntasks; t += G) {
+        if (ti + t >= R.tcap) continue;
+        const uint32_t nv = min(tv, npush - t * tv);
+        task_write(R, ti + t, po + (unsigned long long)t * tv, s_local, ok ? nv : 0u);
+      }
+      if (gtid == 0) {
+        if (!ok || ti + ntasks > R.tcap) {
+          mark_fail(ctl);
+          const unsigned long long lost = ti + ntasks > R.tcap ? ti + ntasks - max(ti, (unsigned long long)R.tcap) : 0;
+          if (lost) atomicAdd(&ctl->outstanding, 0ull - lost);
+        }
+        gc.tail = head + tv;
+      }
+      extra += npush;
+      tail = head + tv;
+      swept = 0;
+      gsync<G>(gi);
+    } else if (tail != *(volatile uint32_t*)&gc.tail) {
+      gsync<G>(gi);
+      if (gtid == 0) gc.tail = tail;
+      gsync<G>(gi);
+    }
+    if (head >= tail) {
+      found = tail + extra - nseed;
+      split_any = extra != 0;
+      dbg_end();
+      return 0;
     }
     if (*(volatile const unsigned int*)R.cancel) {
       gsync<G>(gi);  // every thread has read the control words above
+      found = 0;
       return FLAG_CANCEL;
     }
-    // ---- stage
+    // ---- help the heavy batches of the other sub-groups, then stage
+    if (NSG > 1) {
+      help_others<G, NSG, U>(g, R, ctl, smem, gi, lane, W);
+      gsync<G>(gi);
+    }
+    mark(-1);
     const uint32_t nb = min((uint32_t)G, tail - head);
     uint32_t nq = 0;
     if (gtid < nb) {
       const uint32_t sl = (head + gtid) & (W - 1);
-      unsigned long long e0, e1;
-      uint32_t T;
-      if (rr) {
-        e0 = rr->e0[sl];
-        e1 = e0 + rr->d[sl];
-        T = rr->T[sl];
-      } else {
-        const uint32_t u = ring[sl];
-        e0 = g.off[u];
-        e1 = g.off[u + 1];
-        T = g.thr[u];
-      }
-      if (e1 > e0) {
-        nq = (uint32_t)(((e1 - 1) >> 2) - (e0 >> 2) + 1);
-        rw.q0[gtid] = e0 >> 2;
-        rw.wlo[gtid] = (uint8_t)(e0 & 3);
-        rw.whi[gtid] = (uint8_t)((e1 - 1) & 3);
-        rw.T[gtid] = T;
-      }
-      rw.nq[gtid] = nq;
-      se += e1 - e0;
+      const unsigned long long e0 = me.rr.e0[sl];
+      nq = stage_row<G>(rw, gtid, e0, e0 + me.rr.d[sl], me.rr.T[sl]);
     }
     if (gtid == 0) gc.nlive = 0;
     uint32_t total;
     const uint32_t incl = group_incl_scan<G>(nq, gtid, gi, gc, total);
     if (gtid < nb) rw.qend[gtid] = incl;
     head += nb;  // ring slots [old head, head) are free again: their rows are staged
-    gsync<G>(gi);
-    // ---- sweep: each thread takes U quads per iteration (j, j+G, ..) whose
-    // Philox chains are independent (ILP)
-    int r = -1;
-    uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0;
-    unsigned long long q0_r = 0;
-    for (uint32_t base = 0; base < total; base += U * G) {
-      unsigned long long qk[U];
-      uint32_t Tk[U], mk[U];
-#pragma unroll
-      for (int k = 0; k < U; ++k) {
-        const uint32_t j = base + k * G + gtid;
-        mk[k] = 0u;
-        qk[k] = 0ull;
-        Tk[k] = 0u;
-        if (j < total) {
-          if (j >= qe) {
-            do {
-              ++r;
-              qe = rw.qend[r];
-            } while (j >= qe);
-            nq_r = rw.nq[r];
-            qb = qe - nq_r;
-            q0_r = rw.q0[r];
-            T_r = rw.T[r];
-            wlo_r = rw.wlo[r];
-            whi_r = rw.whi[r];
-          }
-          const uint32_t li = j - qb;
-          uint32_t m = 0xFu;
-          if (li == 0) m &= 0xFu << wlo_r;
-          if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
-          mk[k] = m;
-          qk[k] = q0_r + li;
-          Tk[k] = T_r;
-        }
-      }
-      // all U Philox calls before any branch (independent chains interleave);
-      // one 4-way min per quad against T decides whether the rare exact test runs
-      uint4 wk[U];
-#pragma unroll
-      for (int k = 0; k < U; ++k) wk[k] = philox_at(qk[k], s, TAG_EDGE, K);
-      bool any = false;
-#pragma unroll
-      for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
-      if (!any) continue;
-#pragma unroll
-      for (int k = 0; k < U; ++k) {
-        const uint32_t T = Tk[k];
-        uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
-                        (wk[k].w <= T ? 8u : 0u);
-        live &= mk[k];
-        while (live) {
-          const int i = __ffs(live) - 1;
-          live &= live - 1;
-          const uint32_t v = g.nbr[(qk[k] << 2) + i];
-          const uint32_t p = atomicAdd(&gc.nlive, 1u);
-          if (p < LIVE_CAP) live_v[p] = v;
-          else visit(v);
-        }
-      }
+    // ---- heavy batch: post it as a job the block's warps claim in chunks
+    const bool heavy = NSG > 1 && total >= help_min;
+    const uint32_t ch = 256u;
+    const uint32_t nchunks = heavy ? (total + ch - 1) / ch : 0u;
+    if (heavy && gtid == 0) {
+      Job& j = gc.job;
+      j.total = total;
+      j.nrows = nb;
+      j.s_local = s_local;
+      j.head = head;
+      j.ch = ch;
+      j.done = 0;
+      gc.epoch = (gc.epoch + 1) & 0xFFFFu;
+      __threadfence_block();
+      atomicExch(&j.claim, ((unsigned long long)gc.epoch << 48) | ((unsigned long long)nchunks << 24));
+      __threadfence_block();
+      j.open = 1u;
     }
     gsync<G>(gi);
+    mark(0);
+    // ---- sweep
+    if (heavy) {
+      work_job<G, U>(g, R, ctl, me, lane, W);
+      if (gtid == 0) {
+        gc.job.open = 0;
+        while (*(volatile uint32_t*)&gc.job.done < nchunks) __nanosleep(20);
+        __threadfence_block();
+      }
+    } else {
+      sweep_strided<G, U>(g, R, ctl, me, total, gtid, (uint32_t)s, ctr_hi(s, TAG_EDGE), s_local, head, W);
+    }
+    gsync<G>(gi);
+    mark(1);
     // ---- visit the parked live neighbours, one per thread
     const uint32_t nl = min(*(volatile uint32_t*)&gc.nlive, LIVE_CAP);
-    for (uint32_t t = gtid; t < nl; t += G) visit(live_v[t]);
-    // tail hand-off: once the launch has no new ids left and only a few
-    // samples are still running (the long chains), give this one up; the
-    // host redoes it with a whole SM per sample (tier 2)
-    if (handoff && gtid == 0 && *(volatile const unsigned long long*)&ctl->ticket >= count &&
-        *(volatile const unsigned long long*)&ctl->active <= handoff)
-      atomicOr(&gc.flag, FLAG_HANDOFF);
+#if EIM_PARK_EDGE
+    for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, g.nbr[me.live_e[t]]);
+#else
+    for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, (uint32_t)me.live_e[t]);
+#endif
+    swept += total;
+    nbatch++;
+    nquads += total;
+    nlive_tot += nl;
+    gsync<G>(gi);
+    mark(2);
+  }
+}
+
+// Thread 0 of a sub-group: what to do next.  Tasks first (they belong to
+// the heavy samples that bound the round), then a new sample id; idle while
+// work is outstanding elsewhere (a running traversal may still split); exit
+// when every id is taken and nothing is outstanding.
+__device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
+  const volatile unsigned int* cp = R.cancel;
+  if (cp[0] || cp[1]) return ACT_EXIT;  // cancelled or paused
+  unsigned long long h = vload(&ctl->thead);
+  for (;;) {
+    const unsigned long long t = min(vload(&ctl->ttail), (unsigned long long)R.tcap);
+    if (h >= t) break;
+    const unsigned long long old = atomicCAS(&ctl->thead, h, h + 1);
+    if (old == h) {
+      unsigned long long* d = R.tasks + 2 * h;
+      unsigned long long w1;
+      while ((w1 = vload(d + 1)) == 0ull) __nanosleep(32);  // claimed before it was written
+      __threadfence();
+      gc.base = vload(d);
+      d[0] = 0ull;
+      d[1] = 0ull;  // consumed: the descriptors are all-zero again when the round ends
+      gc.s_local = (uint32_t)(w1 >> 32) - 1u;
+      gc.nb = (uint32_t)w1;
+      return ACT_TASK;
+    }
+    h = old;
+  }
+  if (vload(&ctl->ticket) < count) {
+    atomicAdd(&ctl->outstanding, 1ull);  // before the ticket: an observer never sees "all taken, none outstanding" early
+    const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
+    if (t == 0) ctl->t_first = gtimer();
+    if (t == count - 1) ctl->t_last_id = gtimer();
+    if (t < count) {
+      gc.s_local = (uint32_t)t;
+      gc.nb = 0;
+      return ACT_LOCAL;
+    }
+    atomicAdd(&ctl->outstanding, ~0ull);
+  }
+  if (vload(&ctl->arena_fail)) return ACT_EXIT;  // the host redoes the round
+  if (vload(&ctl->outstanding) == 0ull) {
+    atomicMax(&ctl->t_end, gtimer());
+    return ACT_EXIT;
+  }
+  return ACT_IDLE;
+}
+
+// The IC sampler of one round: persistent blocks of NSG sub-groups over
+// sample ids [0, count) and the tasks split off heavy samples.
+#ifndef EIM_IC_THREADS_SM
+#define EIM_IC_THREADS_SM 1280  // resident sampler threads per SM the register budget is cut for
+#endif
+template <int G, int NSG>
+constexpr int ic_min_blocks() {
+  return EIM_IC_THREADS_SM / (G * NSG) > 0 ? EIM_IC_THREADS_SM / (G * NSG) : 1;
+}
+
+template <int G, int NSG>
+__global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GraphView g, RoundView R, uint64_t count, uint32_t W,
+                                                      SampleCtl* ctl, uint32_t spill_quads, uint32_t task_quads,
+                                                      uint32_t help_min) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int gi = threadIdx.x / G, gtid = threadIdx.x % G, lane = threadIdx.x & 31;
+  const SG<G> me = sg_at<G>(smem_raw, gi, W);
+  GroupCtl& gc = *me.gc;
+  if (gtid == 0) {
+    gc.job.claim = 0;
+    gc.job.open = 0;
+    gc.job.done = 0;
+    gc.epoch = 0;
+  }
+  __syncthreads();  // every sub-group's job is initialised before anyone helps
+  uint32_t backoff = 256;
+  for (;;) {
+    if (gtid == 0) gc.action = decide(R, ctl, count, gc);
+    gsync<G>(gi);
+    const uint32_t act = gc.action;
+    if (act == ACT_EXIT) break;
+    if (act == ACT_IDLE && NSG == 1) {
+      if (gtid == 0) __nanosleep(backoff);
+      backoff = min(backoff * 2u, 2048u);
+    } else if (act == ACT_IDLE) {
+      // poll the block's jobs (shared memory) for ~backoff ns before the
+      // next global poll
+      bool helped = false;
+      const unsigned long long t_end = __shfl_sync(FULL, gtimer(), 0) + backoff;
+      do {
+        helped |= help_others<G, NSG, U_IC>(g, R, ctl, smem_raw, gi, lane, W);
+        __nanosleep(64);
+      } while (__shfl_sync(FULL, gtimer(), 0) < t_end);  // warp-uniform exit
+      backoff = helped ? 256u : min(backoff * 2u, 4096u);
+    } else {
+      backoff = 256;
+      const uint32_t s_local = gc.s_local, nseed = gc.nb;
+      const unsigned long long poff = gc.base;
+      uint32_t found = 0;
+      bool split_any = false;
+      const uint32_t flag = traverse<G, NSG, U_IC>(g, R, ctl, smem_raw, gi, s_local, act == ACT_LOCAL, poff, nseed, W,
+                                                   gtid, found, spill_quads, task_quads, help_min, split_any);
+      if (gtid == 0) {
+        if (found) atomicAdd(&R.sizes[s_local], found);
+        if (split_any && act == ACT_LOCAL) atomicAdd(&ctl->spilled, 1ull);
+        if (flag & FLAG_TABLE) mark_fail(ctl);
+        __threadfence();  // tasks pushed above are counted before this unit leaves `outstanding`
+        atomicAdd(&ctl->outstanding, ~0ull);  // -1
+      }
+    }
     gsync<G>(gi);
   }
 }
 
-// tier 1 (GLOBAL_RING = false): shared-memory ring of W entries per group,
-// over the contiguous ids [0, count).  tier 2 (GLOBAL_RING = true): ring of W
-// entries per group slot in global memory, over a list of failed ids.
-template <int G, bool GLOBAL_RING>
-__global__ void __launch_bounds__(G, (G >= 1024 ? 1 : (G >= 512 ? 2 : 6))) ic_group_kernel(GraphView g, uint64_t seed, RoundView R,
-                                                                        uint64_t count,
-                                                                        const uint32_t* __restrict__ ids,
-                                                                        uint32_t W, SampleCtl* ctl,
-                                                                        uint32_t* retry_out, uint32_t* gring,
-                                                                        uint32_t tier, uint32_t handoff) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const int gi = threadIdx.x / G, gtid = threadIdx.x % G;
-  const size_t per_group = sizeof(GroupCtl) + sizeof(GroupRows<G>) + 4 * LIVE_CAP + (GLOBAL_RING ? 0 : (size_t)20 * W);
-  unsigned char* base = smem_raw + (size_t)gi * per_group;
-  GroupCtl& gc = *reinterpret_cast<GroupCtl*>(base);
-  GroupRows<G>& rw = *reinterpret_cast<GroupRows<G>*>(base + sizeof(GroupCtl));
-  const uint64_t slot = (uint64_t)blockIdx.x * (blockDim.x / G) + gi;
-  unsigned char* dyn = base + sizeof(GroupCtl) + sizeof(GroupRows<G>);
-  uint32_t* live_v = reinterpret_cast<uint32_t*>(dyn);
-  dyn += 4 * LIVE_CAP;
-  uint32_t* ring = GLOBAL_RING ? gring + slot * (uint64_t)W : reinterpret_cast<uint32_t*>(dyn);
-  RingRows rows_smem;
-  if (!GLOBAL_RING) {  // tier 1: ring + prefetched rows in shared memory
-    rows_smem.e0 = reinterpret_cast<unsigned long long*>(dyn + 4ull * W);
-    rows_smem.d = reinterpret_cast<uint32_t*>(dyn + 12ull * W);
-    rows_smem.T = reinterpret_cast<uint32_t*>(dyn + 16ull * W);
-  }
-  const RingRows* rr = GLOBAL_RING ? nullptr : &rows_smem;
-  const PhiloxKey& K = R.K;
-  unsigned long long edges_acc = 0;
-  for (;;) {
-    if (gtid == 0) {
-      // cancelled or paused: take no new id (a resumed launch continues the ticket)
-      const volatile unsigned int* cp = R.cancel;
-      bool stop = cp[0] || cp[1];
-      unsigned long long t = 0;
-      if (!stop) {
-        t = atomicAdd(&ctl->ticket, 1ull);
-        stop = t >= count;
-      }
-      gc.s_local = stop ? 0xFFFFFFFFu : (ids ? ids[t] : (uint32_t)t);
-      if (!stop) atomicAdd(&ctl->active, 1ull);
-    }
-    gsync<G>(gi);
-    const uint32_t s_local = gc.s_local;
-    if (s_local == 0xFFFFFFFFu) break;
-    unsigned long long se = 0;
-    uint32_t size = 0;
-    const uint32_t flag = ic_group_sample<G, IC_U>(g, K, R, s_local, tier, ring, W, rr, live_v, rw, gc, gtid, gi, se,
-                                                       size, ctl, count, handoff);
-    if (gtid == 0) {
-      if (flag == 0) {
-        R.sizes[s_local] = size;
-      } else if (flag & FLAG_TABLE) {
-        atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);  // table too full: host redoes the round
-      } else if (flag & (FLAG_RING | FLAG_HANDOFF)) {
-        R.failed[s_local] = (uint8_t)(tier + 1);  // the next attempt's keys will be the members
-        retry_out[atomicAdd(&ctl->retry_count, 1ull)] = s_local;
-      }
-      atomicAdd(&ctl->active, ~0ull);  // -1
-    }
-    if (flag == 0) {
-      edges_acc += se;
-      unsigned long long ws = se;
-      for (int o = 16; o > 0; o >>= 1) ws += __shfl_xor_sync(FULL, ws, o);
-      if ((threadIdx.x & 31) == 0 && ws) atomicAdd(&R.edges[s_local], ws);
-    }
-    gsync<G>(gi);
-  }
-  for (int o = 16; o > 0; o >>= 1) edges_acc += __shfl_xor_sync(FULL, edges_acc, o);
-  if ((threadIdx.x & 31) == 0 && edges_acc) atomicAdd(&ctl->edges, edges_acc);
+template <int G, int NSG>
+size_t ic_smem(uint32_t W) {
+  return NSG * sg_bytes<G>(W);
 }
 
 // ---------------------------------------------------------------- LT
@@ -390,9 +847,8 @@ __global__ void __launch_bounds__(G, (G >= 1024 ? 1 : (G >= 512 ? 2 : 6))) ic_gr
 // floor(tau * d / 2^32) of u's row (the prefix-scan choice under WC
 // weights); the walk stops when d^-(u) = 0 or the chosen vertex is already in
 // the set.  One thread per walk; visited set = the round table.
-__global__ void __launch_bounds__(256) lt_kernel(GraphView g, uint64_t seed, RoundView R, uint64_t count,
-                                                 SampleCtl* ctl) {
-  const PhiloxKey K = philox_key(seed);
+__global__ void __launch_bounds__(256) lt_kernel(GraphView g, RoundView R, uint64_t count, SampleCtl* ctl) {
+  const PhiloxKey& K = R.K;
   unsigned long long edges_acc = 0;
   for (;;) {
     const volatile unsigned int* cp = R.cancel;
@@ -402,7 +858,7 @@ __global__ void __launch_bounds__(256) lt_kernel(GraphView g, uint64_t seed, Rou
     const uint32_t s_local = (uint32_t)t;
     const uint64_t s = R.base + s_local;
     uint32_t u = draw_root(s, g.n, K);
-    bool ok = table_insert(R.keys, R.bits, table_key(s_local, 0, u)) >= 0;
+    bool ok = table_insert(R.keys, R.bits, table_key(s_local, u)) >= 0;
     uint32_t L = 1;
     unsigned long long steps = 0;
     while (ok) {
@@ -413,7 +869,7 @@ __global__ void __launch_bounds__(256) lt_kernel(GraphView g, uint64_t seed, Rou
       const uint32_t tau = word_of(w, u & 3u);
       const unsigned long long j = __umul64hi((unsigned long long)tau << 32, e1 - e0);
       const uint32_t v = g.nbr[e0 + j];
-      const int ins = table_insert(R.keys, R.bits, table_key(s_local, 0, v));
+      const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
       if (ins == 0) break;
       if (ins < 0) ok = false;
       ++L;
@@ -449,35 +905,32 @@ __global__ void place_sets_kernel(const uint64_t* __restrict__ excl, const uint3
 }
 
 // Every live table entry is a member: arena[start(s) + fill[s]++] = v.
+// IC (off != nullptr): the in-edges examined by a set are exactly the
+// in-edges of its members (each member is expanded once), summed into *esum.
 __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint64_t nslots,
-                               const uint8_t* __restrict__ failed, const uint64_t* __restrict__ set_start,
-                               uint64_t set_index0, uint32_t use, uint32_t* __restrict__ fill,
-                               uint32_t* __restrict__ arena, uint32_t* __restrict__ C) {
+                               const uint64_t* __restrict__ set_start, uint64_t set_index0, uint32_t use,
+                               uint32_t* __restrict__ fill, uint32_t* __restrict__ arena, uint32_t* __restrict__ C,
+                               const uint64_t* __restrict__ off, unsigned long long* __restrict__ esum) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long e = 0;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nslots; i += stride) {
     const unsigned long long k = keys[i];
     if (k == 0ull) continue;
-    const uint32_t hi = (uint32_t)(k >> 32);
-    const uint32_t tier = hi >> 30;
-    const uint32_t s_local = (hi & 0x3FFFFFFFu) - 1u;
-    if (s_local >= use) continue;                // speculative samples beyond the ones kept
-    if (tier != failed[s_local]) continue;       // an abandoned attempt of a sample that was redone
+    const uint32_t s_local = (uint32_t)(k >> 32) - 1u;
+    if (s_local >= use) continue;  // speculative samples beyond the ones kept
     const uint32_t v = (uint32_t)k;
     const uint32_t p = atomicAdd(&fill[s_local], 1u);
     arena[set_start[set_index0 + s_local] + p] = v;
     if (C) atomicAdd(&C[v], 1u);
+    if (off) e += off[v + 1] - off[v];
+  }
+  if (off) {
+    for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(FULL, e, o);
+    if ((threadIdx.x & 31) == 0 && e) atomicAdd(esum, e);
   }
 }
 
-constexpr uint32_t IC_W = 1024;    // shared-memory frontier ring per group
-constexpr int IC_G2 = 1024;        // tier 2: a whole SM per sample (tail hand-off and ring overflow)
-constexpr uint32_t IC_W2 = 4096;   // tier-2 shared-memory ring
-constexpr int IC_G3 = 512;         // tier 3: global ring of capacity >= n (never fails)
-
-template <int G, bool GR>
-size_t ic_smem_per_group(uint32_t W) {
-  return sizeof(GroupCtl) + sizeof(GroupRows<G>) + 4 * LIVE_CAP + (GR ? 0 : (size_t)20 * W);
-}
+constexpr uint32_t IC_W = 1024;  // shared-memory frontier ring per group
 
 }  // namespace
 
@@ -504,64 +957,80 @@ void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
 }
 
 void round_release(Round& rd) {
-  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.failed, &rd.edges, &rd.fill, &rd.retry, &rd.excl, &rd.ctl};
+  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.edges, &rd.fill, &rd.excl, &rd.ctl, &rd.queue, &rd.dbg};
   for (DevBuf* x : b) x->release();
   for (cudaEvent_t& e : rd.ev) {
     if (e) cudaEventDestroy(e);
     e = nullptr;
   }
   rd.launched = false;
+  rd.qdirty = true;
 }
 
-template <int G, bool GR>
-static void launch_ic(eim_ctx* ctx, const eim_graph* g, uint64_t seed, const RoundView& R, uint64_t count,
-                      const uint32_t* ids, uint32_t W, SampleCtl* ctl, uint32_t* retry_out, uint32_t* gring,
-                      uint64_t max_blocks, cudaStream_t st, bool spare_sm_slot, uint32_t tier, uint32_t handoff) {
-  const size_t smem = ic_smem_per_group<G, GR>(W);
-  auto kern = ic_group_kernel<G, GR>;
+static uint32_t env_u32(const char* name, uint32_t dflt) {
+  const char* e = std::getenv(name);
+  return (e && *e) ? (uint32_t)std::strtoul(e, nullptr, 10) : dflt;
+}
+
+// Spill threshold (quads swept by one group before a sample moves to the
+// shared queue) and ring size; EIM_SPILL_QUADS / EIM_RING_W override them
+// (tests force the spill paths with tiny values; 0 = spill only on overflow).
+static uint32_t spill_quads() { return env_u32("EIM_SPILL_QUADS", 8192); }
+static uint32_t task_quads() { return env_u32("EIM_TASK_QUADS", 8192); }
+static uint32_t ring_w() {
+  uint32_t w = env_u32("EIM_RING_W", IC_W);
+  if (w < 32 || (w & (w - 1)) || w > IC_W) fail(EIM_E_INVAL, "EIM_RING_W must be a power of two in [32, 1024]");
+  return w;
+}
+
+static uint32_t help_min() { return env_u32("EIM_HELP_QUADS", 1024); }
+
+template <int G, int NSG>
+static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint64_t count, SampleCtl* ctl,
+                      cudaStream_t st, bool spare_sm_slot) {
+  const uint32_t W = ring_w();
+  const size_t smem = ic_smem<G, NSG>(W);
+  auto kern = ic_kernel<G, NSG>;
   EIM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;
-  EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, G, smem));
-  if (per_sm < 1) fail(EIM_E_CUDA, "sampler tier does not fit on an SM");
+  EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, G * NSG, smem));
+  if (per_sm < 1) fail(EIM_E_CUDA, "sampler does not fit on an SM");
   if (spare_sm_slot && per_sm > 1) per_sm -= 1;
-  uint64_t blocks = (uint64_t)per_sm * ctx->sm_count;
-  blocks = std::max<uint64_t>(1, std::min<uint64_t>(std::min<uint64_t>(blocks, count), max_blocks));
-  kern<<<(uint32_t)blocks, G, smem, st>>>(g->view, seed, R, count, ids, W, ctl, retry_out, gring, tier, handoff);
+  const uint64_t blocks = std::max<uint64_t>(1, (uint64_t)per_sm * ctx->sm_count);
+  kern<<<(uint32_t)blocks, G * NSG, smem, st>>>(g->view, R, count, W, ctl, spill_quads(), task_quads(), help_min());
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
 }
 
-// Tail hand-off threshold of tier 1 (samples still running when the launch
-// has no ids left), off by default: measured on C2 it did not shorten the
-// rounds (a restarted chain costs about what it had left).  EIM_HANDOFF=<n>
-// enables it for experiments.
-static uint32_t handoff_threshold(eim_ctx*) {
-  const char* e = std::getenv("EIM_HANDOFF");
-  return e ? (uint32_t)std::atoi(e) : 0u;
-}
-
 static RoundView round_view(Round& rd) {
-  return RoundView{rd.table.as<unsigned long long>(), rd.bits, rd.sizes.as<uint32_t>(), rd.failed.as<uint8_t>(),
+  return RoundView{rd.table.as<unsigned long long>(),
+                   rd.bits,
+                   rd.sizes.as<uint32_t>(),
                    rd.edges.as<unsigned long long>(),
-                   reinterpret_cast<const unsigned int*>(rd.ctl.as<SampleCtl>() + 1), rd.first,
+                   reinterpret_cast<const unsigned int*>(rd.ctl.as<SampleCtl>() + 1),
+                   rd.first,
+                   rd.queue.as<uint32_t>(),
+                   reinterpret_cast<unsigned long long*>(static_cast<char*>(rd.queue.p) + 4ull * rd.pcap),
+                   rd.pcap,
+                   rd.tcap,
+                   rd.dbg.as<unsigned long long>(),
                    philox_key(rd.seed)};
 }
 
-// one tier-1 sampler launch over rd's remaining ids, bracketed by events
+// one sampler launch over rd's remaining work, bracketed by events
 static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
   if (rd.nlaunch >= Round::MAX_LAUNCH) fail(EIM_E_STATE, "too many sampler launches in one round");
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
   const RoundView R = round_view(rd);
   EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch], st));
   if (rd.model == EIM_IC) {
-    launch_ic<IC_G, false>(ctx, g, rd.seed, R, rd.count, nullptr, IC_W, ctl, rd.retry.as<uint32_t>(), nullptr,
-                           ~0ull, st, spare_sm_slot, 0, handoff_threshold(ctx));
+    launch_ic<IC_G, IC_NSG>(ctx, g, R, rd.count, ctl, st, spare_sm_slot);
   } else {
     int per_sm = 0;
     EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel, 256, 0));
     if (spare_sm_slot && per_sm > 1) per_sm -= 1;
     uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
-    lt_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(g->view, rd.seed, R, rd.count, ctl);
+    lt_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(g->view, R, rd.count, ctl);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
   }
@@ -571,15 +1040,36 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
   rd.launched = true;
 }
 
-// memsets + first tier-1 launch of rd's range on stream st
+// table + queue sizing, memsets and the first launch of rd's range on st
 static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
   const uint64_t count = rd.count;
   rd.table.reserve(8ull << rd.bits, false, st);
   EIM_CUDA(cudaMemsetAsync(rd.table.p, 0, 8ull << rd.bits, st));
-  EIM_CUDA(cudaMemsetAsync(rd.failed.p, 0, count, st));
+  if (rd.model == EIM_IC) {
+    // task pool: half the table's slots (a task seed is a distinct member,
+    // and the table is sized for >= 4x the expected members), descriptors
+    // for half of that.  Consumers zero the descriptors they take, so
+    // only fresh or abandoned memory needs a memset (the pool is written
+    // before its descriptor is published).
+    rd.pcap = 1ull << (rd.bits - 1);
+    rd.tcap = rd.pcap / 2;
+    void* before = rd.queue.p;
+    rd.queue.reserve(4ull * rd.pcap + 16ull * rd.tcap, false, st);
+    if (rd.queue.p != before) rd.qdirty = true;
+    if (rd.qdirty) {
+      EIM_CUDA(cudaMemsetAsync(static_cast<char*>(rd.queue.p) + 4ull * rd.pcap, 0, 16ull * rd.tcap, st));
+      rd.qdirty = false;
+    }
+  } else {
+    rd.pcap = rd.tcap = 0;
+  }
   EIM_CUDA(cudaMemsetAsync(rd.sizes.p, 0, count * sizeof(uint32_t), st));
   EIM_CUDA(cudaMemsetAsync(rd.edges.p, 0, count * sizeof(unsigned long long), st));
   EIM_CUDA(cudaMemsetAsync(rd.ctl.p, 0, sizeof(SampleCtl) + 16, st));
+  if (std::getenv("EIM_DEBUG_TIMELINE")) {
+    rd.dbg.reserve(64 * count, false, st);
+    EIM_CUDA(cudaMemsetAsync(rd.dbg.p, 0, 64 * count, st));
+  }
   rd.nlaunch = 0;
   round_kernel(ctx, g, rd, st, spare_sm_slot);
 }
@@ -612,10 +1102,8 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   rd.model = model;
   rd.hist = hist;
   rd.sizes.reserve(count * sizeof(uint32_t), false, st);
-  rd.failed.reserve(count, false, st);
   rd.edges.reserve(count * sizeof(unsigned long long), false, st);
   rd.fill.reserve(count * sizeof(uint32_t), false, st);
-  rd.retry.reserve(2 * count * sizeof(uint32_t), false, st);  // two retry lists (tier 1 -> 2 -> 3)
   rd.excl.reserve((count + 1) * sizeof(uint64_t), false, st);
   rd.ctl.reserve(sizeof(SampleCtl) + 16, false, st);
   // table capacity: >= 4x the expected members (mean set size of earlier
@@ -633,6 +1121,7 @@ void round_cancel(eim_ctx* ctx, Round& rd) {
   EIM_CUDA(cudaStreamSynchronize(ctx->aux_stream));
   EIM_CUDA(cudaStreamSynchronize(rd.stream));
   rd.launched = false;
+  rd.qdirty = true;  // items may be left in the queue
 }
 
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use) {
@@ -652,57 +1141,39 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   };
   for (int attempt = 0;; ++attempt) {
     int counted = 0;
-    for (;;) {  // until the tier-1 launches have taken every id (a paused round is resumed here)
+    for (;;) {  // until every id is taken and no task is outstanding (a paused round is resumed here)
       EIM_CUDA(cudaStreamWaitEvent(st, rd.ev[2 * rd.nlaunch - 1], 0));
       EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
       EIM_CUDA(cudaStreamSynchronize(st));
-      if (h->ticket >= rd.count || h->arena_fail) break;
+      if ((h->ticket >= rd.count && h->outstanding == 0) || h->arena_fail) break;
       round_resume(ctx, g, rd, st);
     }
     res.kernel_ms += elapsed(counted);
     res.launches += rd.nlaunch - counted;
-    counted = rd.nlaunch;
-    bool table_full = h->arena_fail != 0;
-    // retry tiers over the ids a tier gave up: tier 2 = a whole SM (1024
-    // threads) per sample with a larger shared-memory ring (the long chains
-    // handed off by tier 1, and ring overflows); tier 3 = global-memory ring
-    // of capacity >= n, which cannot overflow
-    uint32_t* lists[2] = {rd.retry.as<uint32_t>(), rd.retry.as<uint32_t>() + rd.count};
-    if (!table_full && h->retry_count > 0)  // a pause that arrived after the last id was taken
-      EIM_CUDA(cudaMemsetAsync(round_flags(rd) + 1, 0, sizeof(unsigned int), st));
-    for (uint32_t tier = 1; !table_full && h->retry_count > 0; ++tier) {
-      if (tier > 2) fail(EIM_E_CUDA, "tier-3 sampler failed with a ring of capacity n");
-      const uint64_t nretry = h->retry_count;
-      res.tier2 += nretry;
-      uint32_t* in = lists[(tier - 1) & 1];
-      uint32_t* out = lists[tier & 1];
-      EIM_CUDA(cudaMemsetAsync(ctl, 0, sizeof(SampleCtl), st));
-      if (rd.nlaunch >= Round::MAX_LAUNCH) fail(EIM_E_STATE, "too many sampler launches in one round");
-      EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch], st));
-      if (tier == 1) {
-        launch_ic<IC_G2, false>(ctx, g, rd.seed, round_view(rd), nretry, in, IC_W2, ctl, out, nullptr,
-                                ctx->sm_count, st, false, 1, 0);
-      } else {
-        uint32_t W3 = 1;
-        while (W3 < g->view.n) W3 <<= 1;
-        uint64_t slots = std::min<uint64_t>(nretry, std::max<uint64_t>(1, (1ull << 30) / (4ull * W3)));
-        slots = std::min<uint64_t>(slots, (uint64_t)ctx->sm_count);
-        ctx->tier_queue.reserve(slots * (uint64_t)W3 * 4, false, st);
-        launch_ic<IC_G3, true>(ctx, g, rd.seed, round_view(rd), nretry, in, W3, ctl, out,
-                               ctx->tier_queue.as<uint32_t>(), slots, st, false, 2, 0);
+    res.spilled += h->spilled;
+    if (std::getenv("EIM_DEBUG_TIMELINE") && rd.model == EIM_IC) {
+      std::fprintf(stderr, "timeline count=%llu ids_taken_us=%.1f tail_us=%.1f tasks=%llu spilled=%llu kernel_ms=%.3f\n",
+                   (unsigned long long)rd.count, (h->t_last_id - h->t_first) * 1e-3, (h->t_end - h->t_last_id) * 1e-3,
+                   h->tasks_pushed, h->spilled, elapsed(counted));
+      std::vector<unsigned long long> d(8 * rd.count);
+      EIM_CUDA(cudaMemcpy(d.data(), rd.dbg.p, d.size() * 8, cudaMemcpyDeviceToHost));
+      std::vector<uint64_t> idx(rd.count);
+      for (uint64_t i = 0; i < rd.count; ++i) idx[i] = i;
+      std::sort(idx.begin(), idx.end(), [&](uint64_t a, uint64_t b) { return d[8 * a + 3] - d[8 * a + 2] > d[8 * b + 3] - d[8 * b + 2]; });
+      for (int j = 0; j < 5 && j < (int)rd.count; ++j) {
+        const unsigned long long* x = &d[8 * idx[j]];
+        const double us = (x[3] - x[2]) * 1e-3, nb = std::max(1.0, (double)x[0]);
+        std::fprintf(stderr, "  s=%llu batches=%llu quads=%llu live=%llu start_us=%.1f dur_us=%.1f us/batch=%.2f "
+                     "stage=%.2f sweep=%.2f visit=%.2f\n",
+                     (unsigned long long)idx[j], x[0], x[1], x[7], (x[2] - h->t_first) * 1e-3, us, us / nb,
+                     x[4] * 1e-3 / nb, x[5] * 1e-3 / nb, x[6] * 1e-3 / nb);
       }
-      EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch + 1], st));
-      rd.nlaunch++;
-      EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
-      EIM_CUDA(cudaStreamSynchronize(st));
-      res.kernel_ms += elapsed(counted);
-      res.launches += rd.nlaunch - counted;
-      counted = rd.nlaunch;
-      table_full = h->arena_fail != 0;
     }
-    if (table_full) {  // rare: redo the whole range with a 4x larger table
+    counted = rd.nlaunch;
+    if (h->arena_fail) {  // rare: redo the whole range with a 4x larger table (and task pool)
       if (attempt >= 4 || rd.bits >= 31) fail(EIM_E_NOMEM, "membership table overflow");
       rd.bits += 2;
+      rd.qdirty = true;
       round_start(ctx, g, rd, st, false);
       continue;
     }
@@ -718,18 +1189,18 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   sizes_to_offsets_kernel<<<grid_for(ctx, use + 1, 256), 256, 0, st>>>(rd.sizes.as<uint32_t>(), use, excl);
   EIM_CUDA(cudaGetLastError());
   size_t tmp = 0, tmp2 = 0;
+  const bool ic = rd.model == EIM_IC;
+  unsigned long long* d_edges_sum = &ctl->edges;  // IC: summed by the scatter; LT: reduced from per-walk steps
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, use + 1, st));
-  unsigned long long* d_edges_sum = reinterpret_cast<unsigned long long*>(ctl) + 2;  // retry_count slot, unused now
-  EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
   ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, use + 1, st));
-  EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
+  else EIM_CUDA(cudaMemsetAsync(d_edges_sum, 0, sizeof(unsigned long long), st));
   EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + use, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-  EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaMemcpyAsync(h_cursor, d_cursor, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   const uint64_t total = h->ticket, cursor = h_cursor[0];
-  res.edges = h->edges;
   ctx->arena.reserve((cursor + total) * sizeof(uint32_t), true, st);
   const uint64_t set_index0 = rd.first - rd.set_base;
   place_sets_kernel<<<grid_for(ctx, use, 256), 256, 0, st>>>(excl, rd.sizes.as<uint32_t>(), use, cursor, set_index0,
@@ -738,15 +1209,17 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   EIM_CUDA(cudaMemsetAsync(rd.fill.p, 0, use * sizeof(uint32_t), st));
   const uint64_t nslots = 1ull << rd.bits;
   scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
-      rd.table.as<unsigned long long>(), nslots, rd.failed.as<uint8_t>(), ctx->set_start.as<uint64_t>(), set_index0,
+      rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
       (uint32_t)use, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(),
-      rd.hist ? ctx->C_total.as<uint32_t>() : nullptr);
+      rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, ic ? g->view.off : nullptr, d_edges_sum);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;
   h_cursor[0] = cursor + total;
   h_cursor[1] = cursor + total;
   EIM_CUDA(cudaMemcpyAsync(d_cursor, h_cursor, 2 * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+  EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
+  res.edges = h->edges;
   ctx->est_mean_size = std::max(1.0, (double)total / (double)use);
   return res;
 }

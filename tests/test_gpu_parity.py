@@ -73,11 +73,39 @@ def test_sample_rrr_C1_all_ids(eim, ctx, graphs, model):
         eim.eim_graph_free(g)
 
 
+# Split modes of the IC sampler (sample.cu): default threshold; a 64-entry
+# ring that splits its backlog into 32-vertex tasks after every batch; no
+# splits, a 32-entry ring whose overflow leaves as one-vertex tasks.
+SPILL_MODES = {"default": {}, "spill_all": {"EIM_SPILL_QUADS": "1", "EIM_TASK_QUADS": "1", "EIM_RING_W": "64"},
+               "ring32": {"EIM_SPILL_QUADS": "0", "EIM_RING_W": "32"}}
+
+
+@pytest.fixture(params=list(SPILL_MODES))
+def spill_mode(request, monkeypatch):
+    for k, v in SPILL_MODES[request.param].items():
+        monkeypatch.setenv(k, v)
+    return request.param
+
+
+def test_spill_modes_C1(eim, ctx, graphs, spill_mode):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 4, 0, 20000)
+        st = eim.eim_get_stats(ctx)
+        if spill_mode == "spill_all":
+            assert st["spilled_samples"] > 0, st["spilled_samples"]
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 4, 2**50 + 3, 333)
+        _imm_equal(eim, ctx, g, off, nbr, 20, 0.3, 1.0, "IC", 4)
+    finally:
+        eim.eim_graph_free(g)
+
+
 @pytest.mark.parametrize("model", ["IC", "LT"])
 @pytest.mark.parametrize("shape", ["empty", "path", "star", "cycle", "bigcycle", "longpath", "rmat_dense"])
-def test_sample_rrr_special_graphs(eim, ctx, model, shape):
-    # bigcycle (every set = V, 3000 > tier-1 queue) and longpath force the
-    # global-memory tiers; rmat_dense has heavy rows and many live edges.
+def test_sample_rrr_special_graphs(eim, ctx, model, shape, spill_mode):
+    # bigcycle (every set = V, 3000 > the shared-memory ring) and longpath
+    # spill to the shared queue; rmat_dense has heavy rows and many live edges.
     off, nbr = {
         "empty": lambda: inputs.empty_graph(100),
         "path": lambda: inputs.path_graph(50),
@@ -171,13 +199,23 @@ def test_invalid_graphs_rejected(eim, ctx):
 
 
 # ---------------------------------------------------------------- full size
-def test_C2_sampled_sets_and_imm(eim, ctx, graphs):
+def test_C2_sampled_sets_and_imm(eim, ctx, graphs, monkeypatch):
     c = inputs.CONFIGS["C2"]
     off, nbr = graphs("C2")
     g = eim.eim_load_graph_csr(ctx, off, nbr)
     try:
         _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 0, 3000)
-        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 98765, 1500)
+        assert eim.eim_get_stats(ctx)["spilled_samples"] > 0  # the heavy samples take the queue path
+        with monkeypatch.context() as mp:
+            mp.setenv("EIM_SPILL_QUADS", "1")
+            mp.setenv("EIM_TASK_QUADS", "1")
+            _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 98765, 1500)
+            assert eim.eim_get_stats(ctx)["spilled_samples"] > 0
+        with monkeypatch.context() as mp:  # ring overflow: one-vertex tasks
+            mp.setenv("EIM_SPILL_QUADS", "0")
+            mp.setenv("EIM_RING_W", "32")
+            _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 5555, 1000)
+            assert eim.eim_get_stats(ctx)["spilled_samples"] > 0
         st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
         assert st["theta"] > 50000
     finally:

@@ -42,7 +42,7 @@ def main():
             res.append(dict(first=first, count=count, kernel_ms=round(st["ms_sample_kernel"], 3),
                             sample_ms=round(st["ms_sample"], 3), call_ms=round(wall, 2),
                             gedge_s=round(st["edges_examined"] / st["ms_sample_kernel"] / 1e6, 1),
-                            edges=st["edges_examined"], tier2=st["tier2_samples"]))
+                            edges=st["edges_examined"], spilled=st["spilled_samples"]))
         out[var] = res
         for r in res:
             print(var, json.dumps(r))

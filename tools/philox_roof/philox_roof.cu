@@ -46,9 +46,37 @@ void run(int sms) {
   cudaFree(out);
 }
 
-int main() {
+// One 256-thread group alone on the GPU (the latency-bound case of a heavy
+// sampler batch): ns per iteration of ILP chains per thread.
+template <int ILP>
+void single() {
+  uint32_t* out;
+  cudaMalloc(&out, 1 << 20);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  const uint32_t iters = 4096;
+  roof<ILP><<<1, 256>>>(1, 16, out);
+  cudaEventRecord(a);
+  roof<ILP><<<1, 256>>>(1, iters, out);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms;
+  cudaEventElapsedTime(&ms, a, b);
+  printf("{\"single_group_ilp\": %d, \"ns_per_iter\": %.1f, \"quads_per_ns\": %.3f}\n", ILP, ms * 1e6 / iters,
+         256.0 * ILP * iters / (ms * 1e6));
+  cudaFree(out);
+}
+
+int main(int argc, char** argv) {
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  if (argc > 1) {  // latency probe
+    single<1>();
+    single<2>();
+    single<4>();
+    return 0;
+  }
   run<1>(sms);
   run<2>(sms);
   run<4>(sms);
