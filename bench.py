@@ -29,9 +29,10 @@ GRAPH_SEED = 1
 RUN_SEED = 1
 # ALU roofline of the IC sampler: every examined in-edge costs
 # one Philox4x32-10 word; the roof is the Philox word rate of this GPU,
-# measured live by tools/philox_roof (20 IMAD.WIDE per call run at a quarter
-# of the issue rate: ~1.38 calls/clk/SM).  Fallback: the committed
-# measurement in profiles/philox_roof.json.
+# measured live by tools/philox_roof (wide multiplies run at a quarter of the
+# issue rate; the sampler's form hoists the sample-constant work of rounds
+# 0-1: 18 instead of 20 per call), the best form counts.  Fallback: the
+# committed measurement in profiles/philox_roof.json.
 PHILOX_PROBE = os.path.join(ROOT, "tools", "philox_roof", "philox_roof")
 
 
@@ -296,7 +297,8 @@ def main():
             "roofline": {"bound": "alu", "kernel": "ic_kernel (IC sampler, incl. split-off tasks)", "achieved": achieved,
                          "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
                          "traffic": traffic,
-                         "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge), "
+                         "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge; best of the plain and "
+                                       "the sampler's hoisted form, tools/philox_roof), "
                                        + peak_src + "; DESIGN.md §6"},
             "cpu_baseline": cb,
             "e2e": {"value": theta_all / (e2e_ms_step / 1e3), "unit": UNIT,

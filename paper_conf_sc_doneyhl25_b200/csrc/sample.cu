@@ -52,10 +52,6 @@ constexpr uint32_t MAX_PROBE = 256;
 #endif
 constexpr int IC_G = EIM_IC_G;      // threads per sub-group (one traversal at a time)
 constexpr int IC_NSG = EIM_IC_NSG;  // sub-groups per block (one block per SM)
-constexpr int U_IC = 2;             // quads per lane per sweep step (independent Philox chains)
-#ifndef EIM_PARK_EDGE
-#define EIM_PARK_EDGE 1  // 1: park live edge ids and load their in-neighbours in the visit phase
-#endif
 
 // ---------------------------------------------------------------- table
 // key = (s_local + 1) << 32 | v ;  0 = empty slot.  The same 64-bit word is
@@ -111,12 +107,13 @@ __device__ __forceinline__ void gsync(int gi) {
 struct Job {
   unsigned long long claim;
   uint32_t done, open;
-  uint32_t total, nrows, s_local, head, ch, pad;
+  uint32_t total, nrows, s_local, head, ch, hoist;
 };
 
 struct GroupCtl {
   uint32_t tail, flag, s_local, nlive;
   uint32_t pushed, action, nb, epoch;  // pushed: this traversal split off a task
+  uint32_t hiq, pad_[3];               // hiq: a staged row reached Philox quads >= 2^32 (no hoisting)
   unsigned long long h, base;
   Job job;
   uint32_t wsum[32];  // one per warp (G <= 1024)
@@ -167,6 +164,7 @@ struct RoundView {
   uint64_t pcap, tcap;           // pool / descriptor capacity
   unsigned long long* dbg;       // [count][8] per root traversal (EIM_DEBUG_TIMELINE), nullable
   PhiloxKey K;                   // round keys of the seed (kernel parameter: read as constant operands)
+  uint32_t nohoist;              // 1: never use the hoisted edge draws (tests exercise the general path)
 };
 
 constexpr uint32_t LIVE_CAP = 512;  // live in-edges parked per batch (more are visited inline)
@@ -274,177 +272,134 @@ __device__ __forceinline__ void visit_for(const GraphView& g, const RoundView& R
   }
 }
 
-// Light batch: the sub-group's G threads sweep all quads of its staged batch,
-// thread t taking quads t, t + G, .. in groups of U independent Philox chains
-// (rows found by an incremental walk over the scan).
-template <int G, int U>
-__device__ __forceinline__ void sweep_strided(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
-                                              uint32_t total, int gtid, uint32_t c2, uint32_t c3, uint32_t s_local,
-                                              uint32_t head, uint32_t W) {
-  const GroupRows<G>& rw = *o.rw;
-  int r = -1;
-  uint32_t qe = 0, qb = 0, nq_r = 0, T_r = 0, wlo_r = 0, whi_r = 0;
-  unsigned long long q0_r = 0;
-  for (uint32_t base = 0; base < total; base += U * G) {
-    unsigned long long qk[U];
-    uint32_t Tk[U], mk[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      const uint32_t j = base + k * G + gtid;
-      mk[k] = 0u;
-      qk[k] = 0ull;
-      Tk[k] = 0u;
-      if (j < total) {
-        if (j >= qe) {
-          do {
-            ++r;
-            qe = rw.qend[r];
-          } while (j >= qe);
-          nq_r = rw.nq[r];
-          qb = qe - nq_r;
-          q0_r = rw.q0[r];
-          T_r = rw.T[r];
-          wlo_r = rw.wlo[r];
-          whi_r = rw.whi[r];
-        }
-        const uint32_t li = j - qb;
-        uint32_t m = 0xFu;
-        if (li == 0) m &= 0xFu << wlo_r;
-        if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
-        mk[k] = m;
-        qk[k] = q0_r + li;
-        Tk[k] = T_r;
-      }
-    }
-    uint4 wk[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) wk[k] = philox((uint32_t)qk[k], (uint32_t)(qk[k] >> 32), c2, c3, R.K);
-    bool any = false;
-#pragma unroll
-    for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
-    if (!any) continue;
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      const uint32_t T = Tk[k];
-      uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
-                      (wk[k].w <= T ? 8u : 0u);
-      live &= mk[k];
-      while (live) {
-        const int i = __ffs(live) - 1;
-        live &= live - 1;
-        const unsigned long long e = (qk[k] << 2) + i;
-#if EIM_PARK_EDGE
-        // park the edge, not its in-neighbour: the visit phase loads them side by side
-        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
-        if (p < LIVE_CAP) o.live_e[p] = e;
-        else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
-#else
-        const uint32_t v = g.nbr[e];
-        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
-        if (p < LIVE_CAP) o.live_e[p] = v;
-        else visit_for<G>(g, R, ctl, o, s_local, head, W, v);
-#endif
-      }
-    }
+// Row cursor over the merged quad space of o's staged batch: merged index j
+// lies in row r (qend[r] - nq[r] <= j < qend[r]); the row's Philox quad is
+// (qhi, qlo) and its IC threshold T.
+struct Cur {
+  uint32_t j, qe, qlo, qhi, T;
+  int r;
+};
+
+template <int G>
+__device__ __forceinline__ void cur_row(const GroupRows<G>& rw, int r, uint32_t j, Cur& c) {
+  c.r = r;
+  c.j = j;
+  c.qe = rw.qend[r];
+  const unsigned long long q = rw.q0[r] + (j - (c.qe - rw.nq[r]));
+  c.qlo = (uint32_t)q;
+  c.qhi = (uint32_t)(q >> 32);
+  c.T = rw.T[r];
+}
+
+// first row with qend > j (rows with no quads have qend equal to their predecessor's)
+template <int G>
+__device__ __forceinline__ void cur_seek(const GroupRows<G>& rw, uint32_t nrows, uint32_t j, Cur& c) {
+  int lo = 0, hi = (int)nrows - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (rw.qend[mid] > j) hi = mid;
+    else lo = mid + 1;
+  }
+  cur_row<G>(rw, lo, j, c);
+}
+
+template <int G>
+__device__ __forceinline__ void cur_step(const GroupRows<G>& rw, Cur& c) {
+  ++c.j;
+  if (++c.qlo == 0u) ++c.qhi;
+  if (c.j == c.qe) {  // past the row: the next row with quads (only called while j < total)
+    int r = c.r + 1;
+    while (rw.qend[r] <= c.j) ++r;
+    cur_row<G>(rw, r, c.j, c);
   }
 }
 
-// One warp sweeps quads [lo, hi) of o's staged batch (nrows rows; sample
-// counter words c2, c3): lane l takes quads lo + l, lo + l + 32, .. in
-// groups of U independent Philox chains; an edge into the row's vertex is
-// live iff its draw <= T (R2); the in-neighbour of a live edge is parked in
-// o's live list (visited directly when the list is full).
-template <int G, int U>
-__device__ __forceinline__ void sweep_chunk(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
-                                            uint32_t nrows, uint32_t lo, uint32_t hi, int lane, uint32_t c2,
-                                            uint32_t c3, uint32_t s_local, uint32_t head, uint32_t W) {
+template <bool HOIST>
+__device__ __forceinline__ uint4 edge_draws(const Cur& c, const EdgeConsts& E, uint32_t c2, uint32_t c3,
+                                            const PhiloxKey& K) {
+  return HOIST ? philox_edge(c.qlo, E, K) : philox(c.qlo, c.qhi, c2, c3, K);
+}
+
+__device__ __forceinline__ uint32_t min4(const uint4& w) { return min(min(w.x, w.y), min(w.z, w.w)); }
+
+// Rare branch: some word of the quad at c is <= T.  Word i is edge
+// e = 4q + i; it belongs to c's row unless the quad is the row's first
+// (i < wlo) or last (i > whi) and straddles a neighbour row.  A live edge is
+// parked in o's live list (visited directly when the list is full).
+template <int G>
+__device__ __forceinline__ void park_live(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                       const Cur& c, uint4 w, uint32_t s_local, uint32_t head, uint32_t W) {
   const GroupRows<G>& rw = *o.rw;
-  // row of the chunk's first quad lo: first r with qend[r] > lo, found by
-  // the warp in two ballots over <= 32 x 8 rows (the lanes then walk on)
-  int r = 0;
-  {
-    const int seg = ((int)nrows + 31) >> 5;  // rows per lane segment (<= 8 for G = 256)
-    const int last = min((lane + 1) * seg, (int)nrows) - 1;
-    const bool past = last >= 0 && last >= lane * seg && rw.qend[last] > lo;
-    const unsigned bal = __ballot_sync(FULL, past);
-    const int L = bal ? __ffs(bal) - 1 : 31;
-    const int r0 = L * seg;
-    const int idx = r0 + lane;
-    const bool p2 = lane < seg && idx < (int)nrows && rw.qend[idx] > lo;
-    const unsigned b2 = __ballot_sync(FULL, p2);
-    r = b2 ? r0 + __ffs(b2) - 1 : (int)nrows - 1;
+  uint32_t live = (w.x <= c.T ? 1u : 0u) | (w.y <= c.T ? 2u : 0u) | (w.z <= c.T ? 4u : 0u) | (w.w <= c.T ? 8u : 0u);
+  if (c.j == c.qe - rw.nq[c.r]) live &= 0xFu << rw.wlo[c.r];
+  if (c.j == c.qe - 1u) live &= 0xFu >> (3u - rw.whi[c.r]);
+  const unsigned long long q = ((unsigned long long)c.qhi << 32) | c.qlo;
+  while (live) {
+    const int i = __ffs(live) - 1;
+    live &= live - 1;
+    const unsigned long long e = (q << 2) + i;
+    const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
+    if (p < LIVE_CAP) o.live_e[p] = e;
+    else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
   }
-  uint32_t qe = rw.qend[r], nq_r = rw.nq[r], qb = qe - nq_r, T_r = rw.T[r], wlo_r = rw.wlo[r], whi_r = rw.whi[r];
-  unsigned long long q0_r = rw.q0[r];
-  for (uint32_t base = lo; base < hi; base += 32 * U) {
-    unsigned long long qk[U];
-    uint32_t Tk[U], mk[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      const uint32_t j = base + k * 32 + lane;
-      mk[k] = 0u;
-      qk[k] = 0ull;
-      Tk[k] = 0u;
-      if (j < hi) {
-        if (j >= qe) {
-          do {
-            ++r;
-            qe = rw.qend[r];
-          } while (j >= qe);
-          nq_r = rw.nq[r];
-          qb = qe - nq_r;
-          q0_r = rw.q0[r];
-          T_r = rw.T[r];
-          wlo_r = rw.wlo[r];
-          whi_r = rw.whi[r];
-        }
-        const uint32_t li = j - qb;
-        uint32_t m = 0xFu;
-        if (li == 0) m &= 0xFu << wlo_r;
-        if (li == nq_r - 1) m &= 0xFu >> (3u - whi_r);
-        mk[k] = m;
-        qk[k] = q0_r + li;
-        Tk[k] = T_r;
-      }
-    }
-    // all U Philox calls before any branch (independent chains interleave);
-    // one 4-way min per quad against T decides whether the rare exact test runs
-    uint4 wk[U];
-#pragma unroll
-    for (int k = 0; k < U; ++k) wk[k] = philox((uint32_t)qk[k], (uint32_t)(qk[k] >> 32), c2, c3, R.K);
-    bool any = false;
-#pragma unroll
-    for (int k = 0; k < U; ++k) any |= (min(min(wk[k].x, wk[k].y), min(wk[k].z, wk[k].w)) <= Tk[k]) & (mk[k] != 0u);
-    if (!any) continue;
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-      const uint32_t T = Tk[k];
-      uint32_t live = (wk[k].x <= T ? 1u : 0u) | (wk[k].y <= T ? 2u : 0u) | (wk[k].z <= T ? 4u : 0u) |
-                      (wk[k].w <= T ? 8u : 0u);
-      live &= mk[k];
-      while (live) {
-        const int i = __ffs(live) - 1;
-        live &= live - 1;
-        const unsigned long long e = (qk[k] << 2) + i;
-#if EIM_PARK_EDGE
-        // park the edge, not its in-neighbour: the visit phase loads them side by side
-        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
-        if (p < LIVE_CAP) o.live_e[p] = e;
-        else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
-#else
-        const uint32_t v = g.nbr[e];
-        const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
-        if (p < LIVE_CAP) o.live_e[p] = v;
-        else visit_for<G>(g, R, ctl, o, s_local, head, W, v);
+}
+
+// NT threads (thread t) sweep quads [lo, hi) of o's staged batch (nrows
+// rows; sample counter words c2, c3): thread t takes one contiguous run and
+// walks it as U interleaved sub-runs (U independent Philox chains in flight).
+// An edge into the row's vertex is live iff its draw <= T (R2); the common
+// case is one 4-way min and one compare per quad.  HOIST: every quad of the
+// batch has qhi = 0, so the sample-constant Philox work is hoisted
+// (philox_edge: 18 instead of 20 wide multiplies per quad).
+#ifndef EIM_SWEEP_U
+#define EIM_SWEEP_U 2
 #endif
-      }
-    }
+template <int G, int NT, bool HOIST, int U>
+__device__ __forceinline__ void sweep_runs(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                           uint32_t nrows, uint32_t lo, uint32_t hi, int t, uint32_t c2, uint32_t c3,
+                                           const EdgeConsts& E, uint32_t s_local, uint32_t head, uint32_t W) {
+  const GroupRows<G>& rw = *o.rw;
+  const uint32_t per = (hi - lo + NT - 1) / NT;
+  const uint32_t a0 = lo + (uint32_t)t * per;
+  if (per == 0 || a0 >= hi) return;
+  const uint32_t a1 = min(a0 + per, hi);
+  const uint32_t sub = (a1 - a0 + U - 1) / U;
+  Cur c[U];
+  uint32_t n[U];
+#pragma unroll
+  for (int k = 0; k < U; ++k) {
+    const uint32_t st = a0 + (uint32_t)k * sub;
+    n[k] = st < a1 ? min(sub, a1 - st) : 0u;
+    if (k == 0 || n[k]) cur_seek<G>(rw, nrows, st, c[k]);
+    else c[k] = c[0];
   }
+  for (uint32_t i = 0;;) {
+    uint4 w[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) w[k] = edge_draws<HOIST>(c[k], E, c2, c3, R.K);
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+      if ((k == 0 || i < n[k]) && min4(w[k]) <= c[k].T) park_live<G>(g, R, ctl, o, c[k], w[k], s_local, head, W);
+    if (++i >= sub) break;
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+      if (k == 0 || i < n[k]) cur_step<G>(rw, c[k]);
+  }
+}
+
+template <int G, int NT>
+__device__ __forceinline__ void sweep_any(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+                                          uint32_t nrows, uint32_t lo, uint32_t hi, int t, uint64_t s,
+                                          uint32_t s_local, uint32_t head, uint32_t W, bool hoist) {
+  const uint32_t c2 = (uint32_t)s, c3 = ctr_hi(s, TAG_EDGE);
+  const EdgeConsts E = edge_consts(0u, c2, c3, R.K);
+  if (hoist) sweep_runs<G, NT, true, EIM_SWEEP_U>(g, R, ctl, o, nrows, lo, hi, t, c2, c3, E, s_local, head, W);
+  else sweep_runs<G, NT, false, 1>(g, R, ctl, o, nrows, lo, hi, t, c2, c3, E, s_local, head, W);
 }
 
 // A warp claims and sweeps chunks of o's current job until none is left.
 // Returns true if it swept anything.
-template <int G, int U>
+template <int G>
 __device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                          int lane, uint32_t W) {
   Job& j = o.gc->job;
@@ -461,10 +416,10 @@ __device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R,
     // the job's fields are stable until this chunk is counted done
     const uint32_t ch = *(volatile uint32_t*)&j.ch, total = *(volatile uint32_t*)&j.total;
     const uint32_t nrows = *(volatile uint32_t*)&j.nrows, s_local = *(volatile uint32_t*)&j.s_local;
-    const uint32_t head = *(volatile uint32_t*)&j.head;
+    const uint32_t head = *(volatile uint32_t*)&j.head, hoist = *(volatile uint32_t*)&j.hoist;
     const uint64_t s = R.base + s_local;
     const uint32_t lo = c * ch, hi = min(lo + ch, total);
-    sweep_chunk<G, U>(g, R, ctl, o, nrows, lo, hi, lane, (uint32_t)s, ctr_hi(s, TAG_EDGE), s_local, head, W);
+    sweep_any<G, 32>(g, R, ctl, o, nrows, lo, hi, lane, s, s_local, head, W, hoist != 0u);
     __syncwarp();
     __threadfence_block();  // parks and ring writes before the chunk counts as done
     if (lane == 0) atomicAdd(&j.done, 1u);
@@ -473,7 +428,7 @@ __device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R,
 }
 
 // Warp-level: join the open jobs of the other sub-groups of the block.
-template <int G, int NSG, int U>
+template <int G, int NSG>
 __device__ __forceinline__ bool help_others(const GraphView& g, const RoundView& R, SampleCtl* ctl,
                                             unsigned char* smem, int gi, int lane, uint32_t W) {
   bool any = false;
@@ -483,7 +438,7 @@ __device__ __forceinline__ bool help_others(const GraphView& g, const RoundView&
     const int o = (gi + k) % NSG;
     const SG<G> so = sg_at<G>(smem, o, W);
     if (!*(volatile uint32_t*)&so.gc->job.open) continue;
-    any |= work_job<G, U>(g, R, ctl, so, lane, W);
+    any |= work_job<G>(g, R, ctl, so, lane, W);
   }
   return any;
 }
@@ -522,7 +477,7 @@ __device__ __forceinline__ uint32_t stage_row(GroupRows<G>& rw, int gtid, unsign
 // the traversals is the unique reachable set of the sampled world, whatever
 // the split.  Returns 0, FLAG_TABLE or FLAG_CANCEL; found = new members
 // inserted by this traversal.
-template <int G, int NSG, int U>
+template <int G, int NSG>
 __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView& R, SampleCtl* ctl,
                                              unsigned char* smem, int gi, uint32_t s_local, bool root,
                                              unsigned long long poff, uint32_t nseed, uint32_t W, int gtid,
@@ -559,6 +514,7 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
   };
   if (gtid == 0) {
     gc.flag = 0;
+    gc.hiq = R.nohoist;
     gc.nlive = 0;
     gc.pushed = 0;
     gc.tail = nseed;
@@ -661,7 +617,7 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
     }
     // ---- help the heavy batches of the other sub-groups, then stage
     if (NSG > 1) {
-      help_others<G, NSG, U>(g, R, ctl, smem, gi, lane, W);
+      help_others<G, NSG>(g, R, ctl, smem, gi, lane, W);
       gsync<G>(gi);
     }
     mark(-1);
@@ -671,11 +627,13 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
       const uint32_t sl = (head + gtid) & (W - 1);
       const unsigned long long e0 = me.rr.e0[sl];
       nq = stage_row<G>(rw, gtid, e0, e0 + me.rr.d[sl], me.rr.T[sl]);
+      if (nq && ((e0 + me.rr.d[sl] - 1) >> 34)) gc.hiq = 1u;  // sticky for the traversal
     }
     if (gtid == 0) gc.nlive = 0;
     uint32_t total;
     const uint32_t incl = group_incl_scan<G>(nq, gtid, gi, gc, total);
     if (gtid < nb) rw.qend[gtid] = incl;
+    const bool hoist = *(volatile uint32_t*)&gc.hiq == 0u;  // written before the scan's barrier
     head += nb;  // ring slots [old head, head) are free again: their rows are staged
     // ---- heavy batch: post it as a job the block's warps claim in chunks
     const bool heavy = NSG > 1 && total >= help_min;
@@ -688,6 +646,7 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
       j.s_local = s_local;
       j.head = head;
       j.ch = ch;
+      j.hoist = hoist ? 1u : 0u;
       j.done = 0;
       gc.epoch = (gc.epoch + 1) & 0xFFFFu;
       __threadfence_block();
@@ -699,24 +658,20 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
     mark(0);
     // ---- sweep
     if (heavy) {
-      work_job<G, U>(g, R, ctl, me, lane, W);
+      work_job<G>(g, R, ctl, me, lane, W);
       if (gtid == 0) {
         gc.job.open = 0;
         while (*(volatile uint32_t*)&gc.job.done < nchunks) __nanosleep(20);
         __threadfence_block();
       }
     } else {
-      sweep_strided<G, U>(g, R, ctl, me, total, gtid, (uint32_t)s, ctr_hi(s, TAG_EDGE), s_local, head, W);
+      sweep_any<G, G>(g, R, ctl, me, nb, 0, total, gtid, s, s_local, head, W, hoist);
     }
     gsync<G>(gi);
     mark(1);
     // ---- visit the parked live neighbours, one per thread
     const uint32_t nl = min(*(volatile uint32_t*)&gc.nlive, LIVE_CAP);
-#if EIM_PARK_EDGE
     for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, g.nbr[me.live_e[t]]);
-#else
-    for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, (uint32_t)me.live_e[t]);
-#endif
     swept += total;
     nbatch++;
     nquads += total;
@@ -812,7 +767,7 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(Gra
       bool helped = false;
       const unsigned long long t_end = __shfl_sync(FULL, gtimer(), 0) + backoff;
       do {
-        helped |= help_others<G, NSG, U_IC>(g, R, ctl, smem_raw, gi, lane, W);
+        helped |= help_others<G, NSG>(g, R, ctl, smem_raw, gi, lane, W);
         __nanosleep(64);
       } while (__shfl_sync(FULL, gtimer(), 0) < t_end);  // warp-uniform exit
       backoff = helped ? 256u : min(backoff * 2u, 4096u);
@@ -822,7 +777,7 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(Gra
       const unsigned long long poff = gc.base;
       uint32_t found = 0;
       bool split_any = false;
-      const uint32_t flag = traverse<G, NSG, U_IC>(g, R, ctl, smem_raw, gi, s_local, act == ACT_LOCAL, poff, nseed, W,
+      const uint32_t flag = traverse<G, NSG>(g, R, ctl, smem_raw, gi, s_local, act == ACT_LOCAL, poff, nseed, W,
                                                    gtid, found, spill_quads, task_quads, help_min, split_any);
       if (gtid == 0) {
         if (found) atomicAdd(&R.sizes[s_local], found);
@@ -930,6 +885,43 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
   }
 }
 
+
+#ifdef EIM_SWEEP_BENCH
+// Development probe (built only with -DEIM_SWEEP_BENCH): one group sweeps a
+// staged batch of nrows rows of d in-edges each, `reps` times with different
+// sample ids; parks live edges (no visit).  Measures the sweep alone.
+template <int G>
+__global__ void __launch_bounds__(G, EIM_IC_THREADS_SM / G) sweep_bench_kernel(GraphView g, RoundView R, SampleCtl* ctl, uint32_t nrows,
+                                                           uint32_t d, uint32_t reps, unsigned long long* out) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const SG<G> me = sg_at<G>(smem_raw, 0, 32);
+  const int gtid = threadIdx.x;
+  uint32_t nq = 0;
+  if (gtid < (int)nrows) {
+    const unsigned long long e0 = (unsigned long long)gtid * d * 3 + 1;  // spaced rows, ragged quads
+    nq = stage_row<G>(*me.rw, gtid, e0, e0 + d, 0xFFFFFFFFu / d);
+  }
+  if (gtid == 0) me.gc->hiq = 0;
+  uint32_t total;
+  const uint32_t incl = group_incl_scan<G>(nq, gtid, 0, *me.gc, total);
+  if (gtid < (int)nrows) me.rw->qend[gtid] = incl;
+  unsigned long long t0 = 0, nl = 0;
+  for (uint32_t r = 0; r < reps; ++r) {
+    if (gtid == 0) me.gc->nlive = 0;
+    gsync<G>(0);
+    if (r == 1 && gtid == 0) t0 = gtimer();
+    sweep_any<G, G>(g, R, ctl, me, nrows, 0, total, gtid, 1000 + r + blockIdx.x * reps, 0, 0, 32, true);
+    gsync<G>(0);
+    nl += min(me.gc->nlive, LIVE_CAP);
+  }
+  if (gtid == 0) {
+    out[3 * blockIdx.x] = gtimer() - t0;
+    out[3 * blockIdx.x + 1] = (unsigned long long)total * (reps - 1);
+    out[3 * blockIdx.x + 2] = nl;
+  }
+}
+#endif
+
 constexpr uint32_t IC_W = 1024;  // shared-memory frontier ring per group
 
 }  // namespace
@@ -1014,7 +1006,8 @@ static RoundView round_view(Round& rd) {
                    rd.pcap,
                    rd.tcap,
                    rd.dbg.as<unsigned long long>(),
-                   philox_key(rd.seed)};
+                   philox_key(rd.seed),
+                   std::getenv("EIM_NO_HOIST") ? 1u : 0u};
 }
 
 // one sampler launch over rd's remaining work, bracketed by events
@@ -1233,3 +1226,32 @@ SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uin
 }
 
 }  // namespace eim
+
+#ifdef EIM_SWEEP_BENCH
+extern "C" int eim_dev_sweep_bench(int blocks, uint32_t nrows, uint32_t d, uint32_t reps, double* ns_per_batch,
+                                   double* quads_per_ns) {
+  using namespace eim;
+  RoundView R{};
+  R.K = philox_key(1);
+  GraphView g{};
+  unsigned long long* out = nullptr;
+  SampleCtl* ctl = nullptr;
+  cudaMalloc(&out, 3 * 8 * blocks);
+  cudaMalloc(&ctl, sizeof(SampleCtl));
+  const size_t smem = sg_bytes<IC_G>(32);
+  cudaFuncSetAttribute(sweep_bench_kernel<IC_G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  for (int it = 0; it < 2; ++it) sweep_bench_kernel<IC_G><<<blocks, IC_G, smem>>>(g, R, ctl, nrows, d, reps, out);
+  std::vector<unsigned long long> h(3 * blocks);
+  cudaMemcpy(h.data(), out, h.size() * 8, cudaMemcpyDeviceToHost);
+  double ns = 0, q = 0;
+  for (int b = 0; b < blocks; ++b) {
+    ns = std::max(ns, (double)h[3 * b]);
+    q += (double)h[3 * b + 1];
+  }
+  *ns_per_batch = ns / (reps - 1);
+  *quads_per_ns = q / ns;
+  cudaFree(out);
+  cudaFree(ctl);
+  return (int)cudaGetLastError();
+}
+#endif

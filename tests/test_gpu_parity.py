@@ -75,9 +75,12 @@ def test_sample_rrr_C1_all_ids(eim, ctx, graphs, model):
 
 # Split modes of the IC sampler (sample.cu): default threshold; a 64-entry
 # ring that splits its backlog into 32-vertex tasks after every batch; no
-# splits, a 32-entry ring whose overflow leaves as one-vertex tasks.
+# splits, a 32-entry ring whose overflow leaves as one-vertex tasks; the
+# un-hoisted Philox path.
 SPILL_MODES = {"default": {}, "spill_all": {"EIM_SPILL_QUADS": "1", "EIM_TASK_QUADS": "1", "EIM_RING_W": "64"},
-               "ring32": {"EIM_SPILL_QUADS": "0", "EIM_RING_W": "32"}}
+               "ring32": {"EIM_SPILL_QUADS": "0", "EIM_RING_W": "32"},
+               # general Philox path (the hoisted edge draws need quad ids < 2^32)
+               "nohoist": {"EIM_NO_HOIST": "1"}}
 
 
 @pytest.fixture(params=list(SPILL_MODES))

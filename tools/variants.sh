@@ -1,7 +1,10 @@
-# Tuning sweep over compile-time sampler variants (run on the GPU box).
-run() { timeout 300 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --e2e-steps 1 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$1', round(d['ms_per_step'],3), round(d['phase_ms']['sample_kernel'],3), d['result']['spilled_samples'])"; }
-for defs in "-DEIM_IC_NSG=1" "-DEIM_IC_NSG=1 -DEIM_PARK_EDGE=1" "-DEIM_IC_NSG=2 -DEIM_IC_THREADS_SM=1024" "-DEIM_IC_NSG=4 -DEIM_IC_THREADS_SM=1024"; do
-  EIM_NVCC_DEFS="$defs" python paper_conf_sc_doneyhl25_b200/_build.py --force > /dev/null
-  for tq in 6144 8192 12288; do EIM_TASK_QUADS=$tq run "[$defs] tq=$tq"; done
+# Tuning sweep over compile-time sampler variants (run on the GPU box):
+#   bash tools/variants.sh "-DEIM_IC_G=512 -DEIM_IC_THREADS_SM=1024" ...
+# For each variant: rebuild libeim.so and time IMM runs on C2 (sampler kernel
+# ms, greedy ms, total ms per run); restore the default build at the end.
+for defs in "$@"; do
+  echo "=== [$defs]"
+  EIM_NVCC_DEFS="$defs" python paper_conf_sc_doneyhl25_b200/_build.py --force > /dev/null || { echo build failed; continue; }
+  timeout 300 python tools/prof_imm.py ${EIM_VARIANT_CFG:-C2} 4 2>&1 | tail -2
 done
 python paper_conf_sc_doneyhl25_b200/_build.py --force > /dev/null
