@@ -135,13 +135,7 @@ void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_
                                                            ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
-  // advance cursor and valid_end
-  unsigned long long* tail = reinterpret_cast<unsigned long long*>(ctx->ctl.as<SampleCtl>() + 1);
-  unsigned long long* h = static_cast<unsigned long long*>(ctx->h_pinned);
-  h[0] = cur + total;
-  h[1] = cur + total;
-  EIM_CUDA(cudaMemcpyAsync(tail, h, 2 * sizeof(unsigned long long), cudaMemcpyHostToDevice, st));
-  EIM_CUDA(cudaStreamSynchronize(st));
+  ctx->arena_used = cur + total;
 }
 
 }  // namespace eim

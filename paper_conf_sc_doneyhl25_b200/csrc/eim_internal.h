@@ -39,19 +39,6 @@ struct GraphView {
   const uint32_t* thr;   // n: IC threshold floor((2^32-1)/d), 0 if d == 0
 };
 
-// Where a sampler writes its sets.
-struct ArenaView {
-  uint32_t* elems;                 // members
-  unsigned long long* cursor;      // next free element
-  unsigned long long* valid_end;   // max end of a successful reservation
-  uint64_t cap;                    // capacity in elements
-  uint64_t* set_start;             // indexed by sample id - set_base
-  uint32_t* set_len;
-  uint64_t set_base;
-  uint32_t* C;                     // coverage histogram (nullable: no histogram)
-};
-
-// Per-launch control block (device memory).
 // Per-launch control block (device memory).  The counters that every group
 // polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
@@ -116,6 +103,7 @@ struct eim_ctx {
   cudaStream_t rstream[2] = {};                 // sampler streams of rounds[0], rounds[1]
   cudaStream_t aux_stream = nullptr;            // cancel-flag writes
   double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
+  uint64_t arena_used = 0;                      // arena elements in use (host is the authority)
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;

@@ -930,18 +930,12 @@ constexpr uint32_t IC_W = 1024;  // shared-memory frontier ring per group
 void arena_reset(eim_ctx* ctx) {
   ctx->arena.reserve(sizeof(uint32_t) * (1u << 22), false, ctx->stream);
   ctx->ctl.reserve(sizeof(SampleCtl) + 2 * sizeof(unsigned long long), false, ctx->stream);
-  // ctl layout: [SampleCtl][cursor][valid_end]
   EIM_CUDA(cudaMemsetAsync(ctx->ctl.p, 0, sizeof(SampleCtl) + 2 * sizeof(unsigned long long), ctx->stream));
   ctx->est_mean_size = 0;
+  ctx->arena_used = 0;
 }
 
-uint64_t arena_cursor(eim_ctx* ctx) {
-  unsigned long long* cur = reinterpret_cast<unsigned long long*>(ctx->ctl.as<SampleCtl>() + 1);
-  unsigned long long v = 0;
-  EIM_CUDA(cudaMemcpyAsync(&v, cur, sizeof(v), cudaMemcpyDeviceToHost, ctx->stream));
-  EIM_CUDA(cudaStreamSynchronize(ctx->stream));
-  return v;
-}
+uint64_t arena_cursor(eim_ctx* ctx) { return ctx->arena_used; }
 
 void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
   ctx->set_start.reserve(num_sets * sizeof(uint64_t), true, ctx->stream);
@@ -1175,8 +1169,6 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   rd.launched = false;
   if (use == 0) return res;
   // ---- sizes -> offsets (sample-id order) -> arena placement -> scatter + histogram
-  unsigned long long* d_cursor = reinterpret_cast<unsigned long long*>(ctx->ctl.as<SampleCtl>() + 1);
-  unsigned long long* h_cursor = reinterpret_cast<unsigned long long*>(h + 1);
   uint64_t* excl = rd.excl.as<uint64_t>();
   ensure_sets(ctx, rd.first + use - rd.set_base);
   sizes_to_offsets_kernel<<<grid_for(ctx, use + 1, 256), 256, 0, st>>>(rd.sizes.as<uint32_t>(), use, excl);
@@ -1191,9 +1183,8 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
   else EIM_CUDA(cudaMemsetAsync(d_edges_sum, 0, sizeof(unsigned long long), st));
   EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + use, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-  EIM_CUDA(cudaMemcpyAsync(h_cursor, d_cursor, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
-  const uint64_t total = h->ticket, cursor = h_cursor[0];
+  const uint64_t total = h->ticket, cursor = ctx->arena_used;
   ctx->arena.reserve((cursor + total) * sizeof(uint32_t), true, st);
   const uint64_t set_index0 = rd.first - rd.set_base;
   place_sets_kernel<<<grid_for(ctx, use, 256), 256, 0, st>>>(excl, rd.sizes.as<uint32_t>(), use, cursor, set_index0,
@@ -1207,9 +1198,7 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
       rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, ic ? g->view.off : nullptr, d_edges_sum);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;
-  h_cursor[0] = cursor + total;
-  h_cursor[1] = cursor + total;
-  EIM_CUDA(cudaMemcpyAsync(d_cursor, h_cursor, 2 * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+  ctx->arena_used = cursor + total;
   EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   res.edges = h->edges;

@@ -34,6 +34,8 @@ namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr int GB = 512;  // threads per block of the greedy kernel
+constexpr uint32_t BIG = 128;      // covered sets with more members are walked by a whole block
+constexpr uint32_t BIG_CAP = 256;  // queued per block and pick (more are walked by their warp)
 
 __global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t* __restrict__ flags) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -41,12 +43,15 @@ __global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t
     flags[i] = (i < n && C[i] > 0u) ? 1u : 0u;
 }
 
-// pos = exclusive scan of flags: candidate index of v
+// pos = exclusive scan of flags: candidate index of v; nc = pos[n].  Writes
+// the candidate list, the vertex -> candidate map, the working counts W
+// (zero-padded to a multiple of 4) and the counts as u64 over [0, n] (zero
+// past nc) for the inverted-index scan.
 __global__ void compact_kernel(const uint32_t* __restrict__ C, const uint32_t* __restrict__ pos, uint32_t n,
-                               uint32_t nc_pad, uint32_t* __restrict__ cand, uint32_t* __restrict__ cidx,
-                               uint32_t* __restrict__ W) {
+                               uint32_t* __restrict__ cand, uint32_t* __restrict__ cidx, uint32_t* __restrict__ W,
+                               uint64_t* __restrict__ cnt64) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  const uint32_t nc = pos[n];
+  const uint32_t nc = pos[n], nc_pad = (nc + 3u) & ~3u;
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
     const uint32_t c = C[v];
     if (c > 0u) {
@@ -54,9 +59,14 @@ __global__ void compact_kernel(const uint32_t* __restrict__ C, const uint32_t* _
       cand[p] = (uint32_t)v;
       cidx[v] = p;
       W[p] = c;
+      cnt64[p] = c;
     }
   }
-  for (uint64_t i = nc + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nc_pad; i += stride) W[i] = 0u;
+  const uint64_t end = max((uint64_t)n + 1, (uint64_t)nc_pad);
+  for (uint64_t i = nc + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < end; i += stride) {
+    if (i <= n) cnt64[i] = 0ull;
+    if (i < nc_pad) W[i] = 0u;
+  }
 }
 
 __global__ void remap_kernel(const uint32_t* __restrict__ arena, uint64_t total, const uint32_t* __restrict__ cidx,
@@ -66,16 +76,12 @@ __global__ void remap_kernel(const uint32_t* __restrict__ arena, uint64_t total,
     arena_c[i] = cidx[arena[i]];
 }
 
-__global__ void count_to_u64_kernel(const uint32_t* __restrict__ W, uint32_t nc, uint64_t* __restrict__ out) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= nc; i += stride)
-    out[i] = i < nc ? (uint64_t)W[i] : 0ull;
-}
-
-// inverted index fill: one warp per set, inv[fill[x]++] = set id (x = candidate index)
+// inverted index fill: one warp per set.  off[x] holds the END of x's list
+// (inclusive scan of counts); each entry is placed at --off[x], so when the
+// fill is done off[x] is the START of x's list (and off[x+1] its end).
 __global__ void invert_kernel(const uint32_t* __restrict__ arena_c, const uint64_t* __restrict__ set_start,
                               const uint32_t* __restrict__ set_len, uint64_t num_sets,
-                              unsigned long long* __restrict__ fill, uint32_t* __restrict__ inv) {
+                              unsigned long long* __restrict__ off, uint32_t* __restrict__ inv) {
   const int lane = threadIdx.x & 31;
   const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
@@ -83,7 +89,7 @@ __global__ void invert_kernel(const uint32_t* __restrict__ arena_c, const uint64
     const uint64_t st = set_start[i];
     const uint32_t L = set_len[i];
     for (uint32_t t = lane; t < L; t += 32) {
-      const unsigned long long p = atomicAdd(&fill[arena_c[st + t]], 1ull);
+      const unsigned long long p = atomicAdd(&off[arena_c[st + t]], ~0ull) - 1ull;
       inv[p] = (uint32_t)i;
     }
   }
@@ -115,7 +121,8 @@ __device__ __forceinline__ unsigned long long block_max(unsigned long long k, un
 }
 
 struct GreedyArgs {
-  uint32_t k, nc_pad;
+  uint32_t k;
+  const uint32_t* nc;           // candidates (device)
   uint32_t* W;                  // working counts per candidate (padded with 0)
   const uint32_t* cand;         // candidate -> vertex (ascending)
   const uint64_t* inv_off;      // nc+1
@@ -141,7 +148,10 @@ __device__ __forceinline__ unsigned long long gtimer_ns() {
 __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   cg::grid_group grid = cg::this_grid();
   __shared__ unsigned long long red[GB / 32];
-  const uint32_t nc4 = a.nc_pad / 4;
+  __shared__ uint32_t big[BIG_CAP];
+  __shared__ uint32_t nbig;
+  if (threadIdx.x == 0) nbig = 0;
+  const uint32_t nc4 = ((*a.nc + 3u) & ~3u) / 4;
   const uint4* W4 = reinterpret_cast<const uint4*>(a.W);
   const int lane = threadIdx.x & 31;
   const uint64_t warp = ((uint64_t)blockIdx.x * GB + threadIdx.x) >> 5;
@@ -183,17 +193,42 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         a.seeds[j] = v;
         a.gains[j] = km >> 32;
       }
-      // ---- cover: one warp per entry of the winner's inverted list
+      // ---- cover: one warp per entry of the winner's inverted list; a
+      // set larger than BIG (the long reverse-BFS sets) is queued and walked
+      // by the whole block afterwards, so no warp walks thousands of members
       const uint64_t lo = a.inv_off[ci], hi = a.inv_off[ci + 1];
       for (uint64_t p = lo + warp; p < hi; p += nwarps) {
         const uint32_t i = a.inv[p];
         if (a.F[i]) continue;  // covered by an earlier pick (ids are unique within one list)
         __syncwarp();
-        if (lane == 0) a.F[i] = 1;
-        const uint64_t st = a.set_start[i];
         const uint32_t L = a.set_len[i];
+        const uint64_t st = a.set_start[i];
+        bool queued = false;
+        if (lane == 0) {
+          a.F[i] = 1;
+          if (L > BIG) {
+            const uint32_t q = atomicAdd(&nbig, 1u);
+            if (q < BIG_CAP) {
+              big[q] = i;
+              queued = true;
+            }
+          }
+        }
+        if (__shfl_sync(FULL, queued, 0)) continue;
+#pragma unroll 4
         for (uint32_t t = lane; t < L; t += 32) atomicSub(&a.W[a.arena_c[st + t]], 1u);
       }
+      __syncthreads();
+      const uint32_t nb = min(nbig, BIG_CAP);
+      for (uint32_t q = 0; q < nb; ++q) {
+        const uint32_t i = big[q];
+        const uint64_t st = a.set_start[i];
+        const uint32_t L = a.set_len[i];
+#pragma unroll 4
+        for (uint32_t t = threadIdx.x; t < L; t += GB) atomicSub(&a.W[a.arena_c[st + t]], 1u);
+      }
+      __syncthreads();
+      if (threadIdx.x == 0) nbig = 0;
     }
     if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 2] = gtimer_ns();
     grid.sync();
@@ -205,48 +240,37 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
                 uint64_t* gains_out) {
   cudaStream_t st = ctx->stream;
-  uint64_t* h64 = static_cast<uint64_t*>(ctx->h_pinned);
   const uint64_t total = arena_cursor(ctx);  // arena elements of sets [0, num_sets)
-  // ---- 1. candidates (C > 0) in ascending id order
+  // ---- 1. candidates (C > 0) in ascending id order; nc stays on the device
+  // (buffers are sized for nc <= n), so nothing here waits for the host
   ctx->inv_fill.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);  // scratch: flags/pos (u32)
   uint32_t* pos = ctx->inv_fill.as<uint32_t>();
   flag_kernel<<<grid_for(ctx, (uint64_t)n + 1, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), n, pos);
   EIM_CUDA(cudaGetLastError());
-  size_t tmp = 0;
+  size_t tmp = 0, tmp2 = 0;
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, pos, pos, (uint64_t)n + 1, st));
-  ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+  ctx->inv_off.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);
+  uint64_t* inv_off = ctx->inv_off.as<uint64_t>();
+  EIM_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
+  ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, pos, pos, (uint64_t)n + 1, st));
-  uint32_t* h32 = reinterpret_cast<uint32_t*>(h64 + 8);
-  EIM_CUDA(cudaMemcpyAsync(h32, pos + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-  EIM_CUDA(cudaStreamSynchronize(st));
-  const uint32_t nc = *h32;
-  const uint32_t nc_pad = (nc + 3u) & ~3u;
-  ctx->cand.reserve((uint64_t)std::max(nc, 1u) * 4, false, st);
+  ctx->cand.reserve((uint64_t)std::max(n, 1u) * 4, false, st);
   ctx->cidx.reserve((uint64_t)n * 4, false, st);
-  ctx->C_work.reserve((uint64_t)std::max(nc_pad, 4u) * 4, false, st);
-  compact_kernel<<<grid_for(ctx, n, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), pos, n, nc_pad,
-                                                          ctx->cand.as<uint32_t>(), ctx->cidx.as<uint32_t>(),
-                                                          ctx->C_work.as<uint32_t>());
+  ctx->C_work.reserve(((uint64_t)n + 4) * 4, false, st);
+  compact_kernel<<<grid_for(ctx, n, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), pos, n, ctx->cand.as<uint32_t>(),
+                                                          ctx->cidx.as<uint32_t>(), ctx->C_work.as<uint32_t>(), inv_off);
   EIM_CUDA(cudaGetLastError());
   // ---- 2. arena in candidate indices + inverted index
   ctx->arena_c.reserve(std::max<uint64_t>(total, 1) * 4, false, st);
   if (total)
     remap_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(ctx->arena.as<uint32_t>(), total, ctx->cidx.as<uint32_t>(),
                                                               ctx->arena_c.as<uint32_t>());
-  ctx->inv_off.reserve(((uint64_t)nc + 1) * sizeof(uint64_t), false, st);
-  uint64_t* inv_off = ctx->inv_off.as<uint64_t>();
-  count_to_u64_kernel<<<grid_for(ctx, (uint64_t)nc + 1, 256), 256, 0, st>>>(ctx->C_work.as<uint32_t>(), nc, inv_off);
-  EIM_CUDA(cudaGetLastError());
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, inv_off, inv_off, (uint64_t)nc + 1, st));
-  ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, inv_off, inv_off, (uint64_t)nc + 1, st));
-  ctx->stage_c.reserve(((uint64_t)nc + 1) * sizeof(uint64_t), false, st);
-  EIM_CUDA(cudaMemcpyAsync(ctx->stage_c.p, inv_off, ((uint64_t)nc + 1) * sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
+  EIM_CUDA(cub::DeviceScan::InclusiveSum(ctx->scratch.p, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
   ctx->inv.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
   if (num_sets > 0 && total > 0) {
     invert_kernel<<<grid_for(ctx, num_sets * 32, 256), 256, 0, st>>>(
         ctx->arena_c.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), num_sets,
-        ctx->stage_c.as<unsigned long long>(), ctx->inv.as<uint32_t>());
+        reinterpret_cast<unsigned long long*>(inv_off), ctx->inv.as<uint32_t>());
     EIM_CUDA(cudaGetLastError());
   }
   // ---- 3. the k picks in one cooperative kernel
@@ -266,7 +290,7 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
   GreedyArgs a;
   a.k = k;
-  a.nc_pad = nc_pad;
+  a.nc = pos + n;
   a.W = ctx->C_work.as<uint32_t>();
   a.cand = ctx->cand.as<uint32_t>();
   a.inv_off = inv_off;
