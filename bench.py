@@ -168,6 +168,8 @@ def main():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--budget-ids", type=int, default=1 << 20,
+                    help="fixed sample budget of the sampler-throughput leg (0: skip)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -236,14 +238,21 @@ def main():
     theta_all = stats[-1]["theta"]
     value = theta_all / (ms_per_step / 1e3)
 
-    # dominant kernel: IC sampler; per-launch duration from CUDA events on the ctx stream
+    # dominant kernel: the sampler; per-launch duration from CUDA events on its stream
     k_ms = sum(s["ms_sample_kernel"] for s in stats)
     k_launch = sum(s["sample_launches"] for s in stats)
     k_edges_local = sum(s["edges_examined"] for s in stats)
-    peak, peak_src = philox_roof_gwords() if rank == 0 else (1630.0, "")
-    achieved = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
+    if c["model"] == "IC":
+        peak, peak_src = philox_roof_gwords() if rank == 0 else (1630.0, "")
+        achieved = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
+    else:
+        # LT walk step: in_off pair (16 B) + the chosen in_nbr (4 B) + one
+        # 8-B membership-table key = 28 algorithmic bytes
+        peak = float(_peaks().get("hbm_gbs", 8000.0))
+        peak_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in _peaks() else "fallback 8 TB/s"
+        achieved = (28.0 * k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
     traffic = None  # DRAM bytes per sampler launch from the committed ncu --set full capture
-    tpath = os.path.join(ROOT, "profiles", "ncu_sampler.json")
+    tpath = os.path.join(ROOT, "profiles", "ncu_sampler.json" if c["model"] == "IC" else "ncu_sampler_lt.json")
     if os.path.exists(tpath):
         try:
             ls = [l for l in json.load(open(tpath))["launches"] if "dram_bytes" in l]
@@ -268,6 +277,24 @@ def main():
         if i > 0:
             e2e_ms.append(dt)
         assert np.array_equal(s2, seeds) and th2 == theta_all
+    # sampler throughput on a fixed sample budget: theta-
+    # independent, so the rate is not masked by the IMM rounds' tails.  This
+    # rank samples its share of ids [0, B); device time of the sampler kernels.
+    budget = None
+    if args.budget_ids > 0:
+        lo_b, hi_b = eim.eim_shard_range(0, args.budget_ids, rank, world)
+        eim.eim_sample_rrr(ctx, g, c["model"], RUN_SEED, lo_b, min(hi_b - lo_b, 4096))  # warm-up
+        eim.eim_sample_rrr(ctx, g, c["model"], RUN_SEED, lo_b, hi_b - lo_b)
+        sb = eim.eim_get_stats(ctx)
+        bt = torch.tensor([sb["ms_sample_kernel"], float(sb["edges_examined"])], dtype=torch.float64, device=dev)
+        if world > 1:
+            bmax = bt[:1].clone()
+            dist.all_reduce(bmax, op=dist.ReduceOp.MAX)
+            dist.all_reduce(bt, op=dist.ReduceOp.SUM)
+            bt[0] = bmax[0]
+        b_ms, b_edges = float(bt[0].item()), float(bt[1].item())
+        budget = {"ids": args.budget_ids, "kernel_ms": b_ms, "sets_per_s": args.budget_ids / (b_ms / 1e3),
+                  "edges_per_s": b_edges / (b_ms / 1e3), "edges": b_edges, "launches": sb["sample_launches"]}
     te = torch.tensor([statistics.mean(e2e_ms) if e2e_ms else float("nan")], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
@@ -294,12 +321,18 @@ def main():
                          "sample_kernel": k_ms / args.steps,
                          "select": sum(s["ms_select"] for s in stats) / args.steps,
                          "comm": sum(s["ms_comm"] for s in stats) / args.steps},
-            "roofline": {"bound": "alu", "kernel": "ic_kernel (IC sampler, incl. split-off tasks)", "achieved": achieved,
-                         "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
-                         "traffic": traffic,
-                         "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge; best of the plain and "
-                                       "the sampler's hoisted form, tools/philox_roof), "
-                                       + peak_src + "; DESIGN.md §6"},
+            "roofline": ({"bound": "alu", "kernel": "ic_kernel (IC sampler, incl. split-off tasks)", "achieved": achieved,
+                          "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
+                          "traffic": traffic,
+                          "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge; best of the "
+                                        "plain and the sampler's hoisted form, tools/philox_roof), "
+                                        + peak_src + "; DESIGN.md §6"} if c["model"] == "IC" else
+                         {"bound": "hbm", "kernel": "lt_kernel (LT reverse walks)", "achieved": achieved,
+                          "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
+                          "traffic": traffic,
+                          "peak_basis": "28 algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
+            "sampler_fixed_budget": (dict(budget, frac=(budget["edges_per_s"] / 1e9 / world / peak)
+                                          if c["model"] == "IC" else None) if budget else None),
             "cpu_baseline": cb,
             "e2e": {"value": theta_all / (e2e_ms_step / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": int(off.nbytes + nbr.nbytes), "d2h_bytes_per_step": int(4 * c["k"] + 16),

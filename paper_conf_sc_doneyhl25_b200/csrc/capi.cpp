@@ -140,6 +140,12 @@ eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint
       EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
       EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
       EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
+      // keep freed stream-ordered memory in the device's pool: reloading a
+      // graph or regrowing a buffer reuses it instead of cudaMalloc/cudaFree
+      cudaMemPool_t pool;
+      EIM_CUDA(cudaDeviceGetDefaultMemPool(&pool, device));
+      uint64_t keep_all = UINT64_MAX;
+      EIM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep_all));
       EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
       EIM_CUDA(cudaEventCreate(&c->ev0));
       EIM_CUDA(cudaEventCreate(&c->ev1));
@@ -164,6 +170,8 @@ void eim_destroy(eim_ctx* ctx) {
   comm_destroy(ctx->comm);
   free_ctx_buffers(ctx);
   cudaFreeHost(ctx->h_pinned);
+  cudaMemPool_t pool;  // hand the pooled memory back
+  if (cudaDeviceGetDefaultMemPool(&pool, ctx->device) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
   cudaEventDestroy(ctx->ev0);
   cudaEventDestroy(ctx->ev1);
   for (cudaStream_t rs : ctx->rstream) {
@@ -190,9 +198,10 @@ eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64
     g->ctx = ctx;
     cudaStream_t st = ctx->stream;
     try {
-      EIM_CUDA(cudaMalloc(&g->d_off, ((uint64_t)n + 1) * sizeof(uint64_t)));
-      EIM_CUDA(cudaMalloc(&g->d_nbr, std::max<uint64_t>(m, 4) * sizeof(uint32_t)));
-      EIM_CUDA(cudaMalloc(&g->d_thr, (uint64_t)n * sizeof(uint32_t)));
+      // stream-ordered from the context's pool (no device-wide sync)
+      EIM_CUDA(cudaMallocAsync(&g->d_off, ((uint64_t)n + 1) * sizeof(uint64_t), st));
+      EIM_CUDA(cudaMallocAsync(&g->d_nbr, std::max<uint64_t>(m, 4) * sizeof(uint32_t), st));
+      EIM_CUDA(cudaMallocAsync(&g->d_thr, (uint64_t)n * sizeof(uint32_t), st));
       EIM_CUDA(cudaMemcpyAsync(g->d_off, in_offsets, ((uint64_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, st));
       if (m) EIM_CUDA(cudaMemcpyAsync(g->d_nbr, in_neighbors, m * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
       g->view.n = n;
@@ -202,10 +211,10 @@ eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64
       g->view.thr = static_cast<const uint32_t*>(g->d_thr);
       graph_validate_and_thresholds(ctx, g);
     } catch (...) {
+      if (g->d_off) cudaFreeAsync(g->d_off, st);
+      if (g->d_nbr) cudaFreeAsync(g->d_nbr, st);
+      if (g->d_thr) cudaFreeAsync(g->d_thr, st);
       cudaStreamSynchronize(st);
-      if (g->d_off) cudaFree(g->d_off);
-      if (g->d_nbr) cudaFree(g->d_nbr);
-      if (g->d_thr) cudaFree(g->d_thr);
       g->magic = 0;
       delete g;
       throw;
@@ -218,12 +227,18 @@ eim_status eim_graph_free(eim_graph* g) {
   if (!g || g->magic != GRAPH_MAGIC) return EIM_E_STATE;
   eim_ctx* ctx = g->ctx;
   if (ctx_ok(ctx)) {
+    // every kernel that reads the graph has finished when a hot-path call
+    // returns (the calls end synchronised), so the free is stream-ordered
     cudaSetDevice(ctx->device);
+    cudaFreeAsync(g->d_off, ctx->stream);
+    cudaFreeAsync(g->d_nbr, ctx->stream);
+    cudaFreeAsync(g->d_thr, ctx->stream);
     cudaStreamSynchronize(ctx->stream);
+  } else {
+    cudaFree(g->d_off);
+    cudaFree(g->d_nbr);
+    cudaFree(g->d_thr);
   }
-  cudaFree(g->d_off);
-  cudaFree(g->d_nbr);
-  cudaFree(g->d_thr);
   g->magic = 0;
   delete g;
   return EIM_OK;
