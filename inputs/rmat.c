@@ -41,14 +41,18 @@ typedef struct {
   uint64_t* keys;  /* (dst << 32) | src */
   uint64_t* idx;   /* attempt index */
   uint64_t cnt;
+  int oom;
 } gen_job;
 
 static void* gen_worker(void* arg) {
   gen_job* j = (gen_job*)arg;
-  uint64_t cap = (j->t1 - j->t0);
-  j->keys = (uint64_t*)malloc((cap ? cap : 1) * sizeof(uint64_t));
-  j->idx = (uint64_t*)malloc((cap ? cap : 1) * sizeof(uint64_t));
+  /* kept attempts are held in buffers grown on demand (not sized by the
+   * attempt count: at C4/C5 that would be ~3x the kept edges) */
+  uint64_t cap = (j->t1 - j->t0) / 4 + 1024;
+  j->keys = (uint64_t*)malloc(cap * sizeof(uint64_t));
+  j->idx = (uint64_t*)malloc(cap * sizeof(uint64_t));
   j->cnt = 0;
+  j->oom = 0;
   for (uint64_t t = j->t0; t < j->t1; ++t) {
     uint32_t src = 0, dst = 0;
     for (uint32_t lvl = 0; lvl < j->s; ++lvl) {
@@ -65,6 +69,14 @@ static void* gen_worker(void* arg) {
     src = j->perm[src];
     dst = j->perm[dst];
     if (src >= j->n || dst >= j->n || src == dst) continue;
+    if (j->cnt == cap) {
+      cap += cap / 2;
+      uint64_t* k2 = (uint64_t*)realloc(j->keys, cap * sizeof(uint64_t));
+      if (k2) j->keys = k2;
+      uint64_t* i2 = k2 ? (uint64_t*)realloc(j->idx, cap * sizeof(uint64_t)) : NULL;
+      if (!i2) { j->oom = 1; return NULL; }
+      j->idx = i2;
+    }
     j->keys[j->cnt] = ((uint64_t)dst << 32) | src;
     j->idx[j->cnt] = t;
     j->cnt++;
@@ -174,10 +186,19 @@ int rmat_generate(uint32_t n, uint64_t m, double a, double b, double c, uint64_t
       pthread_create(&th[t], NULL, gen_worker, j);
     }
     uint64_t total = 0;
-    for (int t = 0; t < nthreads; ++t) { pthread_join(th[t], NULL); total += jobs[t].cnt; }
-    uint64_t* keys = (uint64_t*)malloc((total ? total : 1) * sizeof(uint64_t));
-    uint64_t* idx = (uint64_t*)malloc((total ? total : 1) * sizeof(uint64_t));
-    if (!keys || !idx) return -1;
+    int oom = 0;
+    for (int t = 0; t < nthreads; ++t) {
+      pthread_join(th[t], NULL);
+      total += jobs[t].cnt;
+      oom |= jobs[t].oom || !jobs[t].keys || !jobs[t].idx;
+    }
+    uint64_t* keys = oom ? NULL : (uint64_t*)malloc((total ? total : 1) * sizeof(uint64_t));
+    uint64_t* idx = oom ? NULL : (uint64_t*)malloc((total ? total : 1) * sizeof(uint64_t));
+    if (!keys || !idx) {
+      for (int t = 0; t < nthreads; ++t) { free(jobs[t].keys); free(jobs[t].idx); }
+      free(keys); free(idx); free(jobs); free(th); free(perm);
+      return -1;
+    }
     uint64_t pos = 0;
     for (int t = 0; t < nthreads; ++t) {
       memcpy(keys + pos, jobs[t].keys, jobs[t].cnt * sizeof(uint64_t));

@@ -18,6 +18,9 @@ _SRC = os.path.join(_HERE, "eim_oracle.c")
 _HDR = os.path.join(_HERE, "eim_oracle.h")
 
 IC, LT = 0, 1
+# run flags (eim_oracle.h): source-vertex elimination (NEXT-1), fresh final phase (NEXT-4)
+SOURCE_ELIM, FRESH_FINAL = 1, 2
+FRESH_BASE = 1 << 61
 MODELS = {"IC": IC, "LT": LT, IC: IC, LT: LT}
 
 # -ffp-contract=off / no fast-math: the theta schedule must be evaluated as written.
@@ -38,6 +41,7 @@ class _Arena(ctypes.Structure):
         ("offsets", ctypes.POINTER(ctypes.c_uint64)),
         ("members", ctypes.POINTER(ctypes.c_uint32)),
         ("edges_examined", ctypes.c_uint64),
+        ("set_edges", ctypes.POINTER(ctypes.c_uint64)),
     ]
 
 
@@ -57,6 +61,7 @@ class ImmStats(ctypes.Structure):
         ("cov", ctypes.c_uint64),
         ("edges_examined", ctypes.c_uint64),
         ("arena_elems", ctypes.c_uint64),
+        ("ids_sampled", ctypes.c_uint64),
     ]
 
 
@@ -80,10 +85,12 @@ def _load():
             "orc_lt_choice": (U32, [U32, U64]),
             "orc_rrr_set": (U32, [U32, P, P, I32, U64, U64, P, P]),
             "orc_sample": (ctypes.POINTER(_Arena), [U32, P, P, I32, U64, U64, U64, I32]),
+            "orc_sample_ex": (ctypes.POINTER(_Arena), [U32, P, P, I32, U64, U64, U64, U32, I32]),
             "orc_arena_free": (None, [ctypes.POINTER(_Arena)]),
             "orc_greedy": (U64, [U32, U64, P, P, U32, P, P]),
             "orc_imm_params": (I32, [U32, U32, D, D, ctypes.POINTER(Params)]),
             "orc_imm": (I32, [U32, P, P, U32, D, D, I32, U64, I32, P, P, P, ctypes.POINTER(ImmStats)]),
+            "orc_imm_ex": (I32, [U32, P, P, U32, D, D, I32, U64, U32, I32, P, P, P, ctypes.POINTER(ImmStats)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -147,17 +154,25 @@ def rrr_set(off, nbr, model, seed, s):
     return out[:sz].copy()
 
 
-def sample(off, nbr, model, seed, first, count, nthreads=1):
-    """Returns (offsets u64[count+1], members u32[total], edges_examined)."""
+def sample(off, nbr, model, seed, first, count, nthreads=1, flags=0, per_set_edges=False):
+    """Returns (offsets u64[count+1], members u32[total], edges_examined)
+    (edges_examined as u64[count], one per set, when per_set_edges)."""
     off, nbr = _graph(off, nbr)
     n = off.size - 1
     L = _load()
-    a = L.orc_sample(n, _ptr(off), _ptr(nbr), MODELS[model], seed, first, count, nthreads)
+    if flags:
+        a = L.orc_sample_ex(n, _ptr(off), _ptr(nbr), MODELS[model], seed, first, count, flags, nthreads)
+    else:
+        a = L.orc_sample(n, _ptr(off), _ptr(nbr), MODELS[model], seed, first, count, nthreads)
     A = a.contents
     offsets = np.ctypeslib.as_array(A.offsets, shape=(count + 1,)).copy()
     members = (np.ctypeslib.as_array(A.members, shape=(A.total,)).copy()
                if A.total else np.zeros(0, dtype=np.uint32))
-    ex = int(A.edges_examined)
+    if per_set_edges:
+        ex = (np.ctypeslib.as_array(A.set_edges, shape=(count,)).copy()
+              if count else np.zeros(0, dtype=np.uint64))
+    else:
+        ex = int(A.edges_examined)
     L.orc_arena_free(a)
     return offsets, members, ex
 
@@ -182,16 +197,16 @@ def imm_params(n, k, eps, ell):
     return p
 
 
-def imm(off, nbr, k, eps, ell, model, seed, nthreads=1):
-    """Returns dict(seeds, theta, spread, stats)."""
+def imm(off, nbr, k, eps, ell, model, seed, nthreads=1, flags=0):
+    """Returns dict(seeds, theta, spread, stats).  flags: SOURCE_ELIM | FRESH_FINAL."""
     off, nbr = _graph(off, nbr)
     n = off.size - 1
     seeds = np.zeros(k, dtype=np.uint32)
     theta = ctypes.c_uint64()
     spread = ctypes.c_double()
     st = ImmStats()
-    rc = _load().orc_imm(n, _ptr(off), _ptr(nbr), k, eps, ell, MODELS[model], seed, nthreads,
-                         _ptr(seeds), ctypes.addressof(theta), ctypes.addressof(spread), ctypes.byref(st))
+    rc = _load().orc_imm_ex(n, _ptr(off), _ptr(nbr), k, eps, ell, MODELS[model], seed, flags, nthreads,
+                            _ptr(seeds), ctypes.addressof(theta), ctypes.addressof(spread), ctypes.byref(st))
     if rc != 0:
         raise RuntimeError(f"orc_imm failed rc={rc}")
     rounds = min(st.rounds, 64)
@@ -200,5 +215,5 @@ def imm(off, nbr, k, eps, ell, model, seed, nthreads=1):
         rounds=int(st.rounds), theta_i=[int(x) for x in st.theta_i[:rounds]],
         cov_i=[int(x) for x in st.cov_i[:rounds]], lambda_p=st.lambda_p, lambda_s=st.lambda_s,
         lb=st.lb, cov=int(st.cov), edges_examined=int(st.edges_examined),
-        arena_elems=int(st.arena_elems),
+        arena_elems=int(st.arena_elems), ids_sampled=int(st.ids_sampled),
     )

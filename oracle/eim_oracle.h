@@ -21,6 +21,10 @@
  *                        gains, tie order)
  *   orc_imm_params ..... pinned (mpmath 40-digit evaluation of [22] Eq. 6/9)
  *   orc_imm ............ pinned through its parts + LB/theta recomputation
+ *   source elimination . pinned (set = plain set minus root; closed forms on
+ *                        path/star; enumeration of the retained-set law)
+ *   fresh final phase .. pinned (estimation identical to the plain run;
+ *                        final = greedy over ids from ORC_FRESH_BASE)
  */
 #ifndef EIM_ORACLE_H
 #define EIM_ORACLE_H
@@ -32,6 +36,9 @@ extern "C" {
 
 enum { ORC_IC = 0, ORC_LT = 1 };
 enum { ORC_TAG_EDGE = 0, ORC_TAG_ROOT = 1, ORC_TAG_LT = 2 };
+/* run flags (NEXT rows of SURVEY §8(f); R22, R23) */
+enum { ORC_SOURCE_ELIM = 1, ORC_FRESH_FINAL = 2 };
+#define ORC_FRESH_BASE (1ULL << 61) /* first sample id of a fresh final phase */
 
 /* ---- randomness (reading R1) ---------------------------------------- */
 void     orc_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]);
@@ -59,11 +66,16 @@ typedef struct {
   uint64_t* offsets;    /* num_sets + 1 */
   uint32_t* members;    /* total */
   uint64_t  edges_examined;  /* IC: sum of in-degrees of expanded vertices; LT: walk steps */
+  uint64_t* set_edges;  /* num_sets: the examined edges (walk steps) of each set */
 } orc_arena;
 
 /* nthreads > 1 splits the id range over threads; the result is identical. */
 orc_arena* orc_sample(uint32_t n, const uint64_t* off, const uint32_t* nbr, int model,
                       uint64_t seed, uint64_t first, uint64_t count, int nthreads);
+/* flags & ORC_SOURCE_ELIM: each set without its source (root) vertex,
+ * possibly empty. */
+orc_arena* orc_sample_ex(uint32_t n, const uint64_t* off, const uint32_t* nbr, int model,
+                         uint64_t seed, uint64_t first, uint64_t count, uint32_t flags, int nthreads);
 void       orc_arena_free(orc_arena* a);
 
 /* ---- greedy NodeSelection (Alg. 3) ------------------------- */
@@ -86,11 +98,18 @@ typedef struct {
   uint64_t cov;              /* coverage of the final seed set */
   uint64_t edges_examined;
   uint64_t arena_elems;
+  uint64_t ids_sampled;      /* sample ids drawn (> theta with source elimination) */
 } orc_imm_stats;
 
 int orc_imm(uint32_t n, const uint64_t* off, const uint32_t* nbr, uint32_t k, double eps,
             double ell, int model, uint64_t seed, int nthreads,
             uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, orc_imm_stats* st);
+/* flags: ORC_SOURCE_ELIM | ORC_FRESH_FINAL.  Returns -1 for invalid
+ * parameters, including ORC_SOURCE_ELIM on a graph without an edge u->v,
+ * u != v (every eliminated set would be empty). */
+int orc_imm_ex(uint32_t n, const uint64_t* off, const uint32_t* nbr, uint32_t k, double eps,
+               double ell, int model, uint64_t seed, uint32_t flags, int nthreads,
+               uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, orc_imm_stats* st);
 
 #ifdef __cplusplus
 }
