@@ -91,6 +91,10 @@ def _load():
             "orc_imm_params": (I32, [U32, U32, D, D, ctypes.POINTER(Params)]),
             "orc_imm": (I32, [U32, P, P, U32, D, D, I32, U64, I32, P, P, P, ctypes.POINTER(ImmStats)]),
             "orc_imm_ex": (I32, [U32, P, P, U32, D, D, I32, U64, U32, I32, P, P, P, ctypes.POINTER(ImmStats)]),
+            "orc_log_bits": (U32, [U64]),
+            "orc_log_words": (U64, [U64, U32]),
+            "orc_log_encode": (None, [P, U64, U32, P]),
+            "orc_log_decode": (U64, [P, U64, U32]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -217,3 +221,27 @@ def imm(off, nbr, k, eps, ell, model, seed, nthreads=1, flags=0):
         lb=st.lb, cov=int(st.cov), edges_examined=int(st.edges_examined),
         arena_elems=int(st.arena_elems), ids_sampled=int(st.ids_sampled),
     )
+
+
+def log_bits(x_max):
+    return int(_load().orc_log_bits(int(x_max)))
+
+
+def log_encode(x, b=None):
+    """Log-encode (bit-pack) x: returns (u32 containers, n_b)."""
+    x = np.ascontiguousarray(x, dtype=np.uint64)
+    if b is None:
+        b = log_bits(int(x.max()) if x.size else 0)
+    L = _load()
+    nw = int(L.orc_log_words(x.size, b))
+    w = np.zeros(max(nw, 1), dtype=np.uint32)
+    L.orc_log_encode(_ptr(x) if x.size else None, x.size, b, _ptr(w))
+    return w[:nw], b
+
+
+def log_decode(words, count, b):
+    words = np.ascontiguousarray(words, dtype=np.uint32)
+    if words.size == 0:
+        words = np.zeros(1, dtype=np.uint32)
+    L = _load()
+    return np.array([L.orc_log_decode(_ptr(words), j, b) for j in range(count)], dtype=np.uint64)

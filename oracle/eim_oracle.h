@@ -25,6 +25,8 @@
  *                        path/star; enumeration of the retained-set law)
  *   fresh final phase .. pinned (estimation identical to the plain run;
  *                        final = greedy over ids from ORC_FRESH_BASE)
+ *   orc_log_* .......... pinned (Fig. 1 example, hand-built containers,
+ *                        numpy unpackbits layout, round trip)
  */
 #ifndef EIM_ORACLE_H
 #define EIM_ORACLE_H
@@ -110,6 +112,12 @@ int orc_imm(uint32_t n, const uint64_t* off, const uint32_t* nbr, uint32_t k, do
 int orc_imm_ex(uint32_t n, const uint64_t* off, const uint32_t* nbr, uint32_t k, double eps,
                double ell, int model, uint64_t seed, uint32_t flags, int nthreads,
                uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, orc_imm_stats* st);
+
+/* ---- log encoding (Fig. 1; R19, R24) ------------------------- */
+uint32_t orc_log_bits(uint64_t x_max);                 /* bit_width(x_max) */
+uint64_t orc_log_words(uint64_t count, uint32_t b);    /* 32-bit containers */
+void     orc_log_encode(const uint64_t* x, uint64_t count, uint32_t b, uint32_t* words);
+uint64_t orc_log_decode(const uint32_t* words, uint64_t j, uint32_t b);
 
 #ifdef __cplusplus
 }
