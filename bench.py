@@ -170,6 +170,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--budget-ids", type=int, default=1 << 20,
                     help="fixed sample budget of the sampler-throughput leg (0: skip)")
+    ap.add_argument("--variant-steps", type=int, default=3,
+                    help="timed steps of each NEXT-row variant (log-encoded store, source elimination, "
+                         "fresh final phase); 0: skip")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -280,6 +283,37 @@ def main():
     # sampler throughput on a fixed sample budget: theta-
     # independent, so the rate is not masked by the IMM rounds' tails.  This
     # rank samples its share of ids [0, B); device time of the sampler kernels.
+    # NEXT-row variants: the same IMM with the log-encoded graph
+    # store (NEXT-2), source-vertex elimination (NEXT-1) and the fresh final
+    # phase (NEXT-4); CUDA events on the same stream, L2 flushed between steps.
+    variants = []
+    if args.variant_steps > 0 and world == 1:
+        g_packed = eim.eim_load_graph_csr(ctx, off, nbr, gflags=eim.EIM_G_LOG_ENCODE)
+        for name, gv, flags in (("log_encoded_store", g_packed, 0),
+                                ("source_elim", g, eim.EIM_F_SOURCE_ELIM),
+                                ("source_elim+log_encoded_store", g_packed, eim.EIM_F_SOURCE_ELIM),
+                                ("fresh_final", g, eim.EIM_F_FRESH_FINAL)):
+            for _ in range(2):
+                eim.eim_imm_run(ctx, gv, c["k"], c["eps"], c["ell"], c["model"], RUN_SEED, flags=flags)
+            vms, vst = 0.0, None
+            for _ in range(args.variant_steps):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                vs, vth, vsp, vst = eim.eim_imm_run(ctx, gv, c["k"], c["eps"], c["ell"], c["model"], RUN_SEED,
+                                                    flags=flags)
+                b.record(stream)
+                torch.cuda.synchronize(dev)
+                vms += a.elapsed_time(b)
+            vms /= args.variant_steps
+            variants.append({"variant": name, "ms_per_step": vms, "rrr_sets_per_s": vth / (vms / 1e3),
+                             "theta": vth, "ids_sampled": vst["ids_sampled"], "arena_elems": vst["arena_elems"],
+                             "arena_bytes": 4 * vst["arena_elems"], "graph_bytes": eim.eim_graph_bytes(gv),
+                             "edges_examined": vst["edges_examined"],
+                             "sample_kernel_ms": vst["ms_sample_kernel"], "select_ms": vst["ms_select"],
+                             "seeds_head": vs[:5].tolist(),
+                             "seeds_equal_plain": bool(np.array_equal(vs, seeds)) if flags == 0 else None})
+        eim.eim_graph_free(g_packed)
     budget = None
     if args.budget_ids > 0:
         lo_b, hi_b = eim.eim_shard_range(0, args.budget_ids, rank, world)
@@ -338,6 +372,10 @@ def main():
                     "h2d_bytes_per_step": int(off.nbytes + nbr.nbytes), "d2h_bytes_per_step": int(4 * c["k"] + 16),
                     "ms_per_step": e2e_ms_step},
             "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
+            "memory": {"graph_bytes": eim.eim_graph_bytes(g), "arena_bytes": 4 * stats[-1]["arena_elems"],
+                       "graph_bytes_log_encoded": next((v["graph_bytes"] for v in variants
+                                                        if v["variant"] == "log_encoded_store"), None)},
+            "variants": variants,
             "clocks": clk,
             "result": {"seeds_head": seeds[:10].tolist(), "theta": theta_all, "spread": spread,
                        "rounds": stats[-1]["rounds"], "spilled_samples": stats[-1]["spilled_samples"],

@@ -67,7 +67,24 @@ typedef struct {
   double ms_select;             /* wall time in greedy NodeSelection (incl. index build) */
   double ms_comm;               /* wall time in NCCL exchanges */
   double ms_sample_kernel;      /* device time of the sampler kernels (CUDA events on the ctx stream) */
+  uint64_t ids_sampled;         /* sample ids drawn by the run, all ranks (> theta with EIM_F_SOURCE_ELIM) */
+  uint64_t arena_bytes;         /* device bytes of the stored sets R (log-encoded with an EIM_G_LOG_ENCODE graph) */
 } eim_stats;
+
+/* Run flags of eim_imm_run_ex / eim_sample_rrr_ex. */
+enum {
+  /* Source-vertex elimination (R22): the root of every
+   * RRR set is left out of the stored set.  In eim_imm_run_ex a set left
+   * empty is discarded and does not count toward |R|: R holds the first
+   * theta non-empty sets in sample-id order.  spread_out keeps the method's
+   * n*cov/|R| (biased under elimination, see R22). */
+  EIM_F_SOURCE_ELIM = 1u,
+  /* Fresh final phase ([22]; R23): the final NodeSelection
+   * runs on theta = ceil(lambda* / LB) sets drawn afresh from sample ids
+   * EIM_FRESH_BASE, EIM_FRESH_BASE+1, ... (eim_imm_run_ex only). */
+  EIM_F_FRESH_FINAL = 2u
+};
+#define EIM_FRESH_BASE (1ULL << 61)
 
 /* IMM parameters of [22] (host-only, no device needed). */
 typedef struct {
@@ -116,6 +133,26 @@ eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64
                               const uint32_t* in_neighbors, eim_graph** out);
 eim_status eim_graph_free(eim_graph* g);
 
+/* eim_load_graph_csr_ex: eim_load_graph_csr with graph flags.
+ * EIM_G_LOG_ENCODE (Fig. 1; NEXT-2; R19, R24): after
+ * validation the device store is log-encoded -- in_offsets packed with
+ * bit_width(m) bits per value and in_neighbors with bit_width(max
+ * neighbour) bits, value j at bits [j n_b, (j+1) n_b) of a little-endian
+ * bit stream of 32-bit containers -- and the plain arrays and per-vertex
+ * thresholds are freed; the kernels decode on the fly (T_v recomputed from
+ * the decoded degree).  eim_imm_run / eim_sample_rrr on such a graph also
+ * store the RRR sets R log-encoded, bit_width(n-1) bits per member (P:99:
+ * "applied to both the network data and the RRR sets").  Every result is
+ * identical to the plain store's.
+ * Errors: those of eim_load_graph_csr, EIM_E_INVAL for an unknown flag. */
+enum { EIM_G_LOG_ENCODE = 1u };
+eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                                 const uint32_t* in_neighbors, uint32_t gflags, eim_graph** out);
+/* Device bytes held by the graph store (plain: 8(n+1) + 4 max(m,4) + 4n;
+ * log-encoded: the two container arrays incl. 2 padding words each).
+ * Errors: EIM_E_STATE (freed graph), EIM_E_INVAL (bytes NULL). */
+eim_status eim_graph_bytes(const eim_graph* g, uint64_t* bytes);
+
 /* ---------------------------------------------------------------- IMM
  * eim_imm_run (Alg. 1, with [22] Alg. 2-3): theta estimation by the
  * martingale loop, RRR sampling of sample ids 0..theta-1 (sets are reused
@@ -134,6 +171,17 @@ eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps,
                        eim_model model, uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out,
                        double* spread_out, eim_stats* stats_out);
 
+/* eim_imm_run_ex: eim_imm_run with run flags (EIM_F_SOURCE_ELIM |
+ * EIM_F_FRESH_FINAL; 0 = eim_imm_run).  stats_out->ids_sampled counts the
+ * sample ids drawn.  Errors: those of eim_imm_run, and EIM_E_INVAL for an
+ * unknown flag, EIM_F_SOURCE_ELIM on a multi-GPU context, or
+ * EIM_F_SOURCE_ELIM on a graph with no edge u -> v, u != v (every set would
+ * be empty).
+ */
+eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell,
+                          eim_model model, uint64_t seed, uint32_t flags, uint32_t* seeds_out,
+                          uint64_t* theta_out, double* spread_out, eim_stats* stats_out);
+
 /* eim_sample_rrr (Alg. 2; LT P:134-140): RRR sets of sample ids
  * [first_id, first_id + count), first_id + count <= 2^62, on this context's
  * device (no communication).  Output in sample-id order, each set ascending
@@ -145,6 +193,13 @@ eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps,
 eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
                           uint64_t first_id, uint64_t count, uint64_t* offsets_out,
                           uint32_t* members_out, uint64_t members_cap, uint64_t* members_total);
+/* eim_sample_rrr_ex: flags = 0 or EIM_F_SOURCE_ELIM.  With EIM_F_SOURCE_ELIM
+ * every set is written without its root, possibly empty; the
+ * output still has one set per sample id.  Errors: those of eim_sample_rrr,
+ * EIM_E_INVAL for any other flag. */
+eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
+                             uint64_t first_id, uint64_t count, uint32_t flags, uint64_t* offsets_out,
+                             uint32_t* members_out, uint64_t members_cap, uint64_t* members_total);
 
 /* eim_select_seeds (Alg. 3): greedy max coverage of an arbitrary
  * arena of num_sets sets over vertices [0, n): offsets[num_sets+1]

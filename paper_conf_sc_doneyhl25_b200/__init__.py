@@ -20,13 +20,18 @@ EIM_OK, EIM_E_INVAL, EIM_E_NOMEM, EIM_E_CUDA, EIM_E_NCCL, EIM_E_CAPACITY, EIM_E_
 EIM_IC, EIM_LT = 0, 1
 MODELS = {"IC": EIM_IC, "LT": EIM_LT, EIM_IC: EIM_IC, EIM_LT: EIM_LT}
 NCCL_ID_BYTES = 128
+# run flags (include/eim.h)
+EIM_F_SOURCE_ELIM, EIM_F_FRESH_FINAL = 1, 2
+EIM_FRESH_BASE = 1 << 61
+EIM_G_LOG_ENCODE = 1
 
 STATUS_NAMES = {0: "EIM_OK", -1: "EIM_E_INVAL", -2: "EIM_E_NOMEM", -3: "EIM_E_CUDA", -4: "EIM_E_NCCL",
                 -5: "EIM_E_CAPACITY", -6: "EIM_E_STATE"}
 
 # Every symbol include/eim.h declares (checked by tests/test_abi.py).
 EXPORTS = ["eim_create", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "eim_version",
-           "eim_load_graph_csr", "eim_graph_free", "eim_imm_run", "eim_sample_rrr", "eim_select_seeds",
+           "eim_load_graph_csr", "eim_load_graph_csr_ex", "eim_graph_bytes", "eim_graph_free", "eim_imm_run", "eim_imm_run_ex", "eim_sample_rrr",
+           "eim_sample_rrr_ex", "eim_select_seeds",
            "eim_imm_params", "eim_shard_range", "eim_get_stats"]
 
 
@@ -56,6 +61,8 @@ class Stats(ctypes.Structure):
         ("ms_select", ctypes.c_double),
         ("ms_comm", ctypes.c_double),
         ("ms_sample_kernel", ctypes.c_double),
+        ("ids_sampled", ctypes.c_uint64),
+        ("arena_bytes", ctypes.c_uint64),
     ]
 
     def as_dict(self):
@@ -91,8 +98,12 @@ def lib():
         "eim_version": (ctypes.c_char_p, []),
         "eim_load_graph_csr": (_I, [_P, _U32, _U64, _P, _P, ctypes.POINTER(_P)]),
         "eim_graph_free": (_I, [_P]),
+        "eim_load_graph_csr_ex": (_I, [_P, _U32, _U64, _P, _P, _U32, ctypes.POINTER(_P)]),
+        "eim_graph_bytes": (_I, [_P, ctypes.POINTER(_U64)]),
         "eim_imm_run": (_I, [_P, _P, _U32, _D, _D, _I, _U64, _P, _P, _P, _P]),
+        "eim_imm_run_ex": (_I, [_P, _P, _U32, _D, _D, _I, _U64, _U32, _P, _P, _P, _P]),
         "eim_sample_rrr": (_I, [_P, _P, _I, _U64, _U64, _U64, _P, _P, _U64, _P]),
+        "eim_sample_rrr_ex": (_I, [_P, _P, _I, _U64, _U64, _U64, _U32, _P, _P, _U64, _P]),
         "eim_select_seeds": (_I, [_P, _U32, _U64, _P, _P, _U32, _P, _P]),
         "eim_imm_params": (_I, [_U32, _U32, _D, _D, ctypes.POINTER(ImmParams)]),
         "eim_shard_range": (_I, [_U64, _U64, _I, _I, ctypes.POINTER(_U64), ctypes.POINTER(_U64)]),
@@ -144,15 +155,25 @@ def eim_last_error(ctx=None):
 
 
 # ------------------------------------------------------------------ graph
-def eim_load_graph_csr(ctx, in_offsets, in_neighbors):
-    """in_offsets: u64[n+1] (numpy or pinned torch tensor .numpy()), in_neighbors: u32[m]."""
+def eim_load_graph_csr(ctx, in_offsets, in_neighbors, gflags=0):
+    """in_offsets: u64[n+1] (numpy or pinned torch tensor .numpy()), in_neighbors: u32[m].
+    gflags != 0 (EIM_G_LOG_ENCODE) calls eim_load_graph_csr_ex."""
     off = _host(in_offsets, np.uint64)
     nbr = _host(in_neighbors, np.uint32)
     n = off.size - 1
     out = _P()
-    _check(lib().eim_load_graph_csr(ctx, n, nbr.size, off.ctypes.data, nbr.ctypes.data if nbr.size else None,
-                                    ctypes.byref(out)), ctx)
+    args = (ctx, n, nbr.size, off.ctypes.data, nbr.ctypes.data if nbr.size else None)
+    if gflags:
+        _check(lib().eim_load_graph_csr_ex(*args, gflags, ctypes.byref(out)), ctx)
+    else:
+        _check(lib().eim_load_graph_csr(*args, ctypes.byref(out)), ctx)
     return out.value
+
+
+def eim_graph_bytes(g):
+    b = _U64()
+    _check(lib().eim_graph_bytes(g, ctypes.byref(b)))
+    return int(b.value)
 
 
 def eim_load_graph_csr_ptr(ctx, n, m, off_ptr, nbr_ptr):
@@ -167,26 +188,34 @@ def eim_graph_free(g):
 
 
 # ------------------------------------------------------------------ hot path
-def eim_imm_run(ctx, g, k, eps, ell, model, seed, with_stats=True):
-    """Returns (seeds u32[k], theta, spread, stats dict or None)."""
+def eim_imm_run(ctx, g, k, eps, ell, model, seed, with_stats=True, flags=0):
+    """Returns (seeds u32[k], theta, spread, stats dict or None).  flags != 0 calls eim_imm_run_ex."""
     seeds = np.zeros(k, dtype=np.uint32)
     theta = ctypes.c_uint64()
     spread = ctypes.c_double()
     st = Stats() if with_stats else None
-    _check(lib().eim_imm_run(ctx, g, k, eps, ell, MODELS[model], seed, seeds.ctypes.data, ctypes.addressof(theta),
-                             ctypes.addressof(spread), ctypes.addressof(st) if st is not None else None), ctx)
+    outs = (seeds.ctypes.data, ctypes.addressof(theta), ctypes.addressof(spread),
+            ctypes.addressof(st) if st is not None else None)
+    if flags:
+        _check(lib().eim_imm_run_ex(ctx, g, k, eps, ell, MODELS[model], seed, flags, *outs), ctx)
+    else:
+        _check(lib().eim_imm_run(ctx, g, k, eps, ell, MODELS[model], seed, *outs), ctx)
     return seeds, int(theta.value), float(spread.value), (st.as_dict() if st is not None else None)
 
 
-def eim_sample_rrr(ctx, g, model, seed, first_id, count, members_cap=None):
-    """Returns (offsets u64[count+1], members u32[total]); sets ascending, in sample-id order."""
+def eim_sample_rrr(ctx, g, model, seed, first_id, count, members_cap=None, flags=0):
+    """Returns (offsets u64[count+1], members u32[total]); sets ascending, in sample-id order.
+    flags != 0 (EIM_F_SOURCE_ELIM) calls eim_sample_rrr_ex."""
     offsets = np.zeros(count + 1, dtype=np.uint64)
     total = ctypes.c_uint64()
     cap = members_cap if members_cap is not None else max(16, count * 64)
     while True:
         members = np.zeros(max(cap, 1), dtype=np.uint32)
-        s = lib().eim_sample_rrr(ctx, g, MODELS[model], seed, first_id, count, offsets.ctypes.data,
-                                 members.ctypes.data, cap, ctypes.addressof(total))
+        outs = (offsets.ctypes.data, members.ctypes.data, cap, ctypes.addressof(total))
+        if flags:
+            s = lib().eim_sample_rrr_ex(ctx, g, MODELS[model], seed, first_id, count, flags, *outs)
+        else:
+            s = lib().eim_sample_rrr(ctx, g, MODELS[model], seed, first_id, count, *outs)
         if s == EIM_E_CAPACITY and members_cap is None:
             cap = int(total.value)
             continue

@@ -3,7 +3,7 @@
 // each ascending) and appending sets received from other ranks.
 #include <cub/cub.cuh>
 
-#include "eim_internal.h"
+#include "arena_view.cuh"
 
 namespace eim {
 
@@ -11,7 +11,7 @@ namespace {
 
 
 // One warp per set: C[x] += 1 for every member x (sets have no duplicates).
-__global__ void hist_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,
+__global__ void hist_kernel(const uint32_t* __restrict__ arena, uint32_t ab, const uint64_t* __restrict__ set_start,
                             const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t hi,
                             uint32_t* __restrict__ C) {
   const int lane = threadIdx.x & 31;
@@ -20,7 +20,7 @@ __global__ void hist_kernel(const uint32_t* __restrict__ arena, const uint64_t* 
   for (uint64_t i = lo + warp; i < hi; i += nwarps) {
     const uint64_t st = set_start[i];
     const uint32_t L = set_len[i];
-    for (uint32_t t = lane; t < L; t += 32) atomicAdd(&C[arena[st + t]], 1u);
+    for (uint32_t t = lane; t < L; t += 32) atomicAdd(&C[arena_get(arena, st + t, ab)], 1u);
   }
 }
 
@@ -32,7 +32,7 @@ __global__ void len_to_u64_kernel(const uint32_t* __restrict__ len, uint64_t lo,
 }
 
 // One warp per set: copy arena[set_start[lo+i] ..] to out[offsets[i] ..].
-__global__ void gather_kernel(const uint32_t* __restrict__ arena, const uint64_t* __restrict__ set_start,
+__global__ void gather_kernel(const uint32_t* __restrict__ arena, uint32_t ab, const uint64_t* __restrict__ set_start,
                               const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t count,
                               const uint64_t* __restrict__ offsets, uint32_t* __restrict__ out) {
   const int lane = threadIdx.x & 31;
@@ -41,7 +41,7 @@ __global__ void gather_kernel(const uint32_t* __restrict__ arena, const uint64_t
   for (uint64_t i = warp; i < count; i += nwarps) {
     const uint64_t src = set_start[lo + i], dst = offsets[i];
     const uint32_t L = set_len[lo + i];
-    for (uint32_t t = lane; t < L; t += 32) out[dst + t] = arena[src + t];
+    for (uint32_t t = lane; t < L; t += 32) out[dst + t] = arena_get(arena, src + t, ab);
   }
 }
 
@@ -56,12 +56,20 @@ __global__ void place_kernel(const uint64_t* __restrict__ offsets, uint64_t coun
   }
 }
 
+// Append encoded: arena element base + j <- members[j].
+__global__ void put_kernel(const uint32_t* __restrict__ members, uint64_t total, uint32_t* arena, uint32_t ab,
+                           uint64_t base) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < total; j += stride)
+    arena_put(arena, base + j, ab, members[j]);
+}
+
 }  // namespace
 
 void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi) {
   if (hi <= lo) return;
   hist_kernel<<<grid_for(ctx, (hi - lo) * 32, 256), 256, 0, ctx->stream>>>(
-      ctx->arena.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, hi,
+      ctx->arena.as<uint32_t>(), ctx->arena_b, ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, hi,
       ctx->C_total.as<uint32_t>());
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
@@ -88,7 +96,8 @@ static uint64_t compact_sets(eim_ctx* ctx, uint64_t lo, uint64_t count, bool sor
   uint32_t* out = ctx->stage_b.as<uint32_t>();
   if (count > 0) {
     gather_kernel<<<grid_for(ctx, count * 32, 256), 256, 0, st>>>(
-        ctx->arena.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, count, offs, out);
+        ctx->arena.as<uint32_t>(), ctx->arena_b, ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo,
+        count, offs, out);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
   }
@@ -126,11 +135,16 @@ void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_
   if (count == 0) return;
   ensure_sets(ctx, base + count);
   uint64_t cur = arena_cursor(ctx);
-  const uint64_t cap = ctx->arena.bytes / sizeof(uint32_t);
-  if (cur + total > cap) ctx->arena.reserve(std::max<uint64_t>(cap * 2, cur + total) * sizeof(uint32_t), true, st);
-  if (total)
+  arena_ensure(ctx, cur + total);
+  if (total && ctx->arena_b == 32)
     EIM_CUDA(cudaMemcpyAsync(ctx->arena.as<uint32_t>() + cur, d_members, total * sizeof(uint32_t),
                              cudaMemcpyDeviceToDevice, st));
+  else if (total) {
+    put_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(d_members, total, ctx->arena.as<uint32_t>(), ctx->arena_b,
+                                                          cur);
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches++;
+  }
   place_kernel<<<grid_for(ctx, count, 256), 256, 0, st>>>(d_offsets, count, base, cur,
                                                            ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
   EIM_CUDA(cudaGetLastError());

@@ -186,9 +186,15 @@ void eim_destroy(eim_ctx* ctx) {
 
 eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
                               const uint32_t* in_neighbors, eim_graph** out) {
+  return eim_load_graph_csr_ex(ctx, n, m, in_offsets, in_neighbors, 0u, out);
+}
+
+eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                                 const uint32_t* in_neighbors, uint32_t gflags, eim_graph** out) {
   if (!ctx_ok(ctx)) return EIM_E_STATE;
   return guarded(ctx, [&] {
     if (!out) fail(EIM_E_INVAL, "out is NULL");
+    if (gflags & ~(uint32_t)EIM_G_LOG_ENCODE) fail(EIM_E_INVAL, "unknown graph flag");
     *out = nullptr;
     if (n < 2 || n >= 0xFFFFFFFFu) fail(EIM_E_INVAL, "n must be in [2, 2^32-1)");
     if (m >= (1ull << 40)) fail(EIM_E_INVAL, "m must be < 2^40");
@@ -210,10 +216,15 @@ eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64
       g->view.nbr = static_cast<const uint32_t*>(g->d_nbr);
       g->view.thr = static_cast<const uint32_t*>(g->d_thr);
       graph_validate_and_thresholds(ctx, g);
+      g->bytes = ((uint64_t)n + 1) * sizeof(uint64_t) + std::max<uint64_t>(m, 4) * sizeof(uint32_t) +
+                 (uint64_t)n * sizeof(uint32_t);
+      if (gflags & EIM_G_LOG_ENCODE) graph_log_encode(ctx, g);
     } catch (...) {
       if (g->d_off) cudaFreeAsync(g->d_off, st);
       if (g->d_nbr) cudaFreeAsync(g->d_nbr, st);
       if (g->d_thr) cudaFreeAsync(g->d_thr, st);
+      if (g->d_offw) cudaFreeAsync(g->d_offw, st);
+      if (g->d_nbrw) cudaFreeAsync(g->d_nbrw, st);
       cudaStreamSynchronize(st);
       g->magic = 0;
       delete g;
@@ -230,17 +241,22 @@ eim_status eim_graph_free(eim_graph* g) {
     // every kernel that reads the graph has finished when a hot-path call
     // returns (the calls end synchronised), so the free is stream-ordered
     cudaSetDevice(ctx->device);
-    cudaFreeAsync(g->d_off, ctx->stream);
-    cudaFreeAsync(g->d_nbr, ctx->stream);
-    cudaFreeAsync(g->d_thr, ctx->stream);
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw})
+      if (p) cudaFreeAsync(p, ctx->stream);
     cudaStreamSynchronize(ctx->stream);
   } else {
-    cudaFree(g->d_off);
-    cudaFree(g->d_nbr);
-    cudaFree(g->d_thr);
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw})
+      if (p) cudaFree(p);
   }
   g->magic = 0;
   delete g;
+  return EIM_OK;
+}
+
+eim_status eim_graph_bytes(const eim_graph* g, uint64_t* bytes) {
+  if (!g || g->magic != GRAPH_MAGIC) return EIM_E_STATE;
+  if (!bytes) return EIM_E_INVAL;
+  *bytes = g->bytes;
   return EIM_OK;
 }
 
@@ -252,15 +268,22 @@ static void check_graph(eim_ctx* ctx, const eim_graph* g) {
 eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
                        uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
                        eim_stats* stats_out) {
+  return eim_imm_run_ex(ctx, g, k, eps, ell, model, seed, 0u, seeds_out, theta_out, spread_out, stats_out);
+}
+
+eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
+                          uint64_t seed, uint32_t flags, uint32_t* seeds_out, uint64_t* theta_out,
+                          double* spread_out, eim_stats* stats_out) {
   if (!ctx_ok(ctx)) return EIM_E_STATE;
   return guarded(ctx, [&] {
     check_graph(ctx, g);
+    if (flags & ~(uint32_t)(EIM_F_SOURCE_ELIM | EIM_F_FRESH_FINAL)) fail(EIM_E_INVAL, "unknown flag");
     if (!seeds_out) fail(EIM_E_INVAL, "seeds_out is NULL");
     if (k == 0 || k > g->view.n) fail(EIM_E_INVAL, "k must be in [1, n]");
     if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
     if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
-    imm_run(ctx, g, k, eps, ell, model, seed, seeds_out, theta_out, spread_out, &ctx->last_stats);
+    imm_run(ctx, g, k, eps, ell, model, seed, flags, seeds_out, theta_out, spread_out, &ctx->last_stats);
     if (stats_out) *stats_out = ctx->last_stats;
   });
 }
@@ -268,24 +291,34 @@ eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps,
 eim_status eim_sample_rrr(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first_id,
                           uint64_t count, uint64_t* offsets_out, uint32_t* members_out, uint64_t members_cap,
                           uint64_t* members_total) {
+  return eim_sample_rrr_ex(ctx, g, model, seed, first_id, count, 0u, offsets_out, members_out, members_cap,
+                           members_total);
+}
+
+eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first_id,
+                             uint64_t count, uint32_t flags, uint64_t* offsets_out, uint32_t* members_out,
+                             uint64_t members_cap, uint64_t* members_total) {
   if (!ctx_ok(ctx)) return EIM_E_STATE;
   eim_status cap_status = EIM_OK;
   eim_status s = guarded(ctx, [&] {
     check_graph(ctx, g);
+    if (flags & ~(uint32_t)EIM_F_SOURCE_ELIM) fail(EIM_E_INVAL, "unknown flag");
     if (!offsets_out || !members_total) fail(EIM_E_INVAL, "NULL output");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
     if (first_id + count < first_id || first_id + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids must be < 2^62");
     cudaStream_t st = ctx->stream;
     const auto t0 = std::chrono::steady_clock::now();
     const uint64_t launches0 = ctx->kernel_launches;
-    arena_reset(ctx);
-    const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false);
+    arena_reset(ctx, g->packed ? bit_width((uint64_t)g->view.n - 1) : 32u);
+    const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false,
+                                        (flags & EIM_F_SOURCE_ELIM) ? RF_DROP_ROOT : 0u);
     std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
     ctx->last_stats.edges_examined = r.edges;
     ctx->last_stats.spilled_samples = r.spilled;
     ctx->last_stats.sample_launches = r.launches;
     ctx->last_stats.ms_sample_kernel = r.kernel_ms;
     ctx->last_stats.theta = count;
+    ctx->last_stats.ids_sampled = count;
     ctx->last_stats.ms_sample = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     uint64_t* d_off = nullptr;
     uint32_t* d_mem = nullptr;

@@ -39,6 +39,19 @@ struct GraphView {
   const uint32_t* thr;   // n: IC threshold floor((2^32-1)/d), 0 if d == 0
 };
 
+// Log-encoded reverse CSR (NEXT-2; layout R24): offsets and
+// in-neighbours bit-packed with n_b = bit_width(max) bits each, in 32-bit
+// containers (two zero words of padding so a decode may read 3 words).  No
+// threshold array: T_v = floor((2^32-1)/d) is recomputed from the decoded
+// degree once per expanded vertex.
+struct PackedGraphView {
+  uint32_t n;
+  uint64_t m;
+  const uint32_t* offw;  // n+1 values of boff bits
+  const uint32_t* nbrw;  // m values of bnbr bits
+  uint32_t boff, bnbr;
+};
+
 // Per-launch control block (device memory).  The counters that every group
 // polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
@@ -51,7 +64,8 @@ struct SampleCtl {
   unsigned long long spilled;                   // samples that split off tasks
   unsigned long long tasks_pushed;              // tasks split off
   unsigned long long t_first, t_last_id, t_end;  // %globaltimer: first id taken, last id taken, last group exit (timeline)
-  unsigned long long pad4[9];
+  unsigned long long consumed;                   // source elimination: ids up to the last kept set
+  unsigned long long pad4[8];
 };
 
 struct Comm;  // NCCL communicator wrapper (comm.cpp)
@@ -59,8 +73,14 @@ struct Comm;  // NCCL communicator wrapper (comm.cpp)
 // One sampler launch over sample ids [first, first+count): its membership
 // table and per-sample scratch.  Two of them let the IMM driver sample the
 // next round speculatively while the greedy of the current round runs.
+// Round output flags: source elimination (R22) drops each sample's root from
+// its set; with RF_DROP_EMPTY the sets left empty are discarded and only
+// the first `use` non-empty sets (in sample-id order) are kept.
+enum : uint32_t { RF_DROP_ROOT = 1u, RF_DROP_EMPTY = 2u };
+
 struct Round {
   DevBuf table, sizes, edges, fill, excl, ctl;  // ctl: SampleCtl + cancel/pause flags
+  DevBuf roots, kidx, ksizes;                    // source elimination: roots, kept-set index, kept sizes
   DevBuf dbg;                                    // EIM_DEBUG_TIMELINE per-sample records
   DevBuf queue;                                  // IC task pool (u32 seeds) + descriptors (all-zero between rounds)
   uint64_t first = 0, count = 0, set_base = 0, seed = 0, pcap = 0, tcap = 0;
@@ -73,6 +93,7 @@ struct Round {
   int nlaunch = 0;
   bool launched = false;
   bool hist = true;
+  uint32_t rflags = 0;
 };
 
 }  // namespace eim
@@ -84,6 +105,12 @@ struct eim_graph {
   void* d_off = nullptr;
   void* d_nbr = nullptr;
   void* d_thr = nullptr;
+  bool packed = false;           // log-encoded store (EIM_G_LOG_ENCODE): pview, d_offw, d_nbrw
+  eim::PackedGraphView pview{};
+  void* d_offw = nullptr;
+  void* d_nbrw = nullptr;
+  uint64_t bytes = 0;            // device bytes of the store
+  int proper_edge = -1;  // has an edge u -> v, u != v (1/0; -1 = not yet computed)
 };
 
 struct eim_ctx {
@@ -104,6 +131,7 @@ struct eim_ctx {
   cudaStream_t aux_stream = nullptr;            // cancel-flag writes
   double est_mean_size = 0;                     // mean set size of earlier rounds (table sizing)
   uint64_t arena_used = 0;                      // arena elements in use (host is the authority)
+  uint32_t arena_b = 32;                        // bits per arena element: 32 plain, else log-encoded (R24)
   // per-graph vectors
   eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
   eim::DevBuf best, seeds, gains;
@@ -123,6 +151,9 @@ constexpr uint32_t SENTINEL = 0xFFFFFFFFu;
 
 // ---- graph.cu
 void graph_validate_and_thresholds(eim_ctx* ctx, eim_graph* g);
+// Replace the plain store by its log encoding (frees off/nbr/thr).
+void graph_log_encode(eim_ctx* ctx, eim_graph* g);
+bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g);
 
 // ---- sample.cu
 struct SampleResult {
@@ -130,18 +161,22 @@ struct SampleResult {
   uint64_t spilled = 0;   // samples finished in the shared frontier queue
   uint32_t launches = 0;
   double kernel_ms = 0;
+  uint64_t kept = 0;      // sets appended to the arena
+  uint64_t consumed = 0;  // sample ids used (> kept when empty sets are dropped)
 };
 // Samples ids [first, first+count) into ctx->arena; set index = id - set_base.
 // Histogram into C when hist is true.  (= round_launch + round_finalize)
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
-                          uint64_t first, uint64_t count, uint64_t set_base, bool hist);
+                          uint64_t first, uint64_t count, uint64_t set_base, bool hist, uint32_t rflags = 0);
 // Launch the sampler for ids [first, first+count) into rd on stream st (no
 // host synchronisation).  spare_sm_slot: leave one block slot per SM free
 // (for a concurrent greedy kernel).
 void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first,
-                  uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot);
+                  uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot,
+                  uint32_t rflags = 0);
 // Wait for rd, redo what overflowed, and append its first `use` sets to the
-// arena (sample-id order) with their histogram.
+// arena (sample-id order) with their histogram.  With RF_DROP_EMPTY, `use`
+// is the number of non-empty sets wanted (res.kept <= use, res.consumed ids).
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use);
 // Stop a launched speculative round and wait for it.
 void round_cancel(eim_ctx* ctx, Round& rd);
@@ -150,7 +185,14 @@ void round_cancel(eim_ctx* ctx, Round& rd);
 void round_pause(eim_ctx* ctx, Round& rd);
 void round_resume(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st);
 void round_release(Round& rd);
-void arena_reset(eim_ctx* ctx);
+// Empty the arena; b = bits per element (32: plain u32; < 32: log-encoded,
+// P:99-101, layout R24, written with atomicOr so concurrent writers of one
+// container are safe -- the "thread-safe log encoding" of P:99).
+void arena_reset(eim_ctx* ctx, uint32_t b = 32);
+// Capacity for `elems` elements (contents kept; new containers zeroed when encoded).
+void arena_ensure(eim_ctx* ctx, uint64_t elems);
+inline uint64_t arena_words(uint64_t elems, uint32_t b) { return (elems * b + 31) / 32 + 2; }
+uint32_t bit_width(uint64_t x);
 void ensure_sets(eim_ctx* ctx, uint64_t num_sets);
 uint64_t arena_cursor(eim_ctx* ctx);
 
@@ -172,7 +214,7 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
 // ---- imm.cpp
 void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);
 void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
-             uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
+             uint64_t seed, uint32_t flags, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
              eim_stats* st);
 
 // ---- comm.cpp

@@ -2,7 +2,9 @@
 // weights).  Weights are never stored: under weighted cascade every in-edge of
 // v shares p = 1/d^-(v), so one integer threshold per vertex,
 // T_v = floor((2^32-1)/d), decides liveness as draw <= T_v (reading R2).
-#include "eim_internal.h"
+
+
+#include "graph_view.cuh"
 
 namespace eim {
 
@@ -34,7 +36,125 @@ __global__ void threshold_kernel(const uint64_t* __restrict__ off, uint32_t n, u
   }
 }
 
+// Any edge u -> v with u != v?  A warp per row; stops early once found.
+template <class GV>
+__global__ void proper_edge_kernel(GV g, uint32_t n, unsigned int* found) {
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t v = warp; v < n; v += nwarps) {
+    if (*(volatile unsigned int*)found) return;
+    unsigned int f = 0;
+    const uint64_t e1 = g_off(g, v + 1);
+    for (uint64_t e = g_off(g, v) + lane; e < e1 && !f; e += 32) f = g_nbr(g, e) != (uint32_t)v;
+    if (__any_sync(0xFFFFFFFFu, f)) {
+      if (lane == 0) atomicOr(found, 1u);
+      return;
+    }
+  }
+}
+
+// Log encoding (layout R24): container i holds stream bits
+// [32 i, 32 i + 32); one thread per container ORs in the values that overlap
+// it, so no two threads write the same word.  Containers past the data (the
+// padding) are zero.
+template <class T>
+__global__ void log_encode_kernel(const T* __restrict__ x, uint64_t count, uint32_t b, uint32_t* __restrict__ w,
+                                  uint64_t nwords) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t data_words = (count * b + 31) / 32;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nwords; i += stride) {
+    uint32_t word = 0;
+    if (i < data_words) {
+      const uint64_t t0 = 32 * i;
+      const uint64_t j0 = t0 / b, j1 = min((t0 + 31) / b, count - 1);
+      for (uint64_t j = j0; j <= j1; ++j) {
+        const int64_t sh = (int64_t)(j * b) - (int64_t)t0;  // value j starts at bit sh of this word
+        const uint64_t v = (uint64_t)x[j];
+        word |= (uint32_t)(sh >= 0 ? (v << sh) : (v >> -sh));
+      }
+    }
+    w[i] = word;
+  }
+}
+
+__global__ void max_of_kernel(const uint32_t* __restrict__ x, uint64_t count, unsigned int* out) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  uint32_t m = 0;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) m = max(m, x[i]);
+  for (int o = 16; o > 0; o >>= 1) m = max(m, __shfl_xor_sync(0xFFFFFFFFu, m, o));
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
+}
+
 }  // namespace
+
+uint32_t bit_width(uint64_t x) {
+  uint32_t b = 0;
+  while (b < 64 && (x >> b) != 0) b++;
+  return b;
+}
+
+void graph_log_encode(eim_ctx* ctx, eim_graph* g) {
+  cudaStream_t st = ctx->stream;
+  const uint32_t n = g->view.n;
+  const uint64_t m = g->view.m;
+  // n_b = bit_width(x_max) (R19): offsets top out at m; neighbours at their max
+  ctx->scratch.reserve(1 << 20, false, st);
+  unsigned int* d_max = reinterpret_cast<unsigned int*>(ctx->scratch.p);
+  EIM_CUDA(cudaMemsetAsync(d_max, 0, sizeof(unsigned int), st));
+  if (m) max_of_kernel<<<grid_for(ctx, m, 256), 256, 0, st>>>(g->view.nbr, m, d_max);
+  EIM_CUDA(cudaGetLastError());
+  unsigned int* h = static_cast<unsigned int*>(ctx->h_pinned);
+  EIM_CUDA(cudaMemcpyAsync(h, d_max, sizeof(unsigned int), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+  const uint32_t boff = bit_width(m), bnbr = bit_width(*h);
+  const uint64_t woff = ((uint64_t)(n + 1) * boff + 31) / 32 + 2, wnbr = (m * bnbr + 31) / 32 + 2;
+  EIM_CUDA(cudaMallocAsync(&g->d_offw, woff * sizeof(uint32_t), st));
+  EIM_CUDA(cudaMallocAsync(&g->d_nbrw, wnbr * sizeof(uint32_t), st));
+  log_encode_kernel<uint64_t><<<grid_for(ctx, woff, 256), 256, 0, st>>>(g->view.off, (uint64_t)n + 1, boff,
+                                                                        static_cast<uint32_t*>(g->d_offw), woff);
+  EIM_CUDA(cudaGetLastError());
+  if (bnbr)
+    log_encode_kernel<uint32_t><<<grid_for(ctx, wnbr, 256), 256, 0, st>>>(g->view.nbr, m, bnbr,
+                                                                          static_cast<uint32_t*>(g->d_nbrw), wnbr);
+  else
+    EIM_CUDA(cudaMemsetAsync(g->d_nbrw, 0, wnbr * sizeof(uint32_t), st));
+  EIM_CUDA(cudaGetLastError());
+  ctx->kernel_launches += 3;
+  g->pview = PackedGraphView{n, m, static_cast<const uint32_t*>(g->d_offw), static_cast<const uint32_t*>(g->d_nbrw),
+                             boff, bnbr};
+  g->packed = true;
+  // the plain store is gone: only the packed view may be used from here on
+  EIM_CUDA(cudaFreeAsync(g->d_off, st));
+  EIM_CUDA(cudaFreeAsync(g->d_nbr, st));
+  EIM_CUDA(cudaFreeAsync(g->d_thr, st));
+  g->d_off = g->d_nbr = g->d_thr = nullptr;
+  g->view.off = nullptr;
+  g->view.nbr = nullptr;
+  g->view.thr = nullptr;
+  g->bytes = (woff + wnbr) * sizeof(uint32_t);
+  EIM_CUDA(cudaStreamSynchronize(st));
+}
+
+// Source elimination needs a graph on which some set can be non-empty (R22).
+bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g) {
+  if (g->proper_edge < 0) {
+    cudaStream_t st = ctx->stream;
+    ctx->scratch.reserve(1 << 20, false, st);
+    unsigned int* d = reinterpret_cast<unsigned int*>(ctx->scratch.p);
+    EIM_CUDA(cudaMemsetAsync(d, 0, sizeof(unsigned int), st));
+    const uint32_t grid = grid_for(ctx, (uint64_t)g->view.n * 32, 256);
+    if (g->packed) proper_edge_kernel<<<grid, 256, 0, st>>>(g->pview, g->view.n, d);
+    else proper_edge_kernel<<<grid, 256, 0, st>>>(g->view, g->view.n, d);
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches += 1;
+    unsigned int* h = static_cast<unsigned int*>(ctx->h_pinned);
+    EIM_CUDA(cudaMemcpyAsync(h, d, sizeof(unsigned int), cudaMemcpyDeviceToHost, st));
+    EIM_CUDA(cudaStreamSynchronize(st));
+    const_cast<eim_graph*>(g)->proper_edge = *h ? 1 : 0;
+  }
+  return g->proper_edge == 1;
+}
 
 void graph_validate_and_thresholds(eim_ctx* ctx, eim_graph* g) {
   cudaStream_t st = ctx->stream;

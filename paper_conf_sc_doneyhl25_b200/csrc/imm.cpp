@@ -46,14 +46,15 @@ struct Exchange {
   DevBuf counts, offs_recv, mem_recv, len_send;
 };
 
-// Sample ids [R, R_new) across ranks; afterwards every rank holds all of them.
-void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t R, uint64_t R_new,
-                  eim_stats* st, Exchange& ex) {
+// Sets [R, R_new) (sample ids id_base + set index) across ranks; afterwards
+// every rank holds all of them.
+void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t id_base, uint64_t R,
+                  uint64_t R_new, eim_stats* st, Exchange& ex) {
   const auto t0 = clk::now();
   cudaStream_t s = ctx->stream;
   uint64_t lo, hi;
   eim_shard_range(R, R_new - R, ctx->rank, ctx->world, &lo, &hi);
-  SampleResult r = sample_range(ctx, g, model, seed, lo, hi - lo, 0, false);
+  SampleResult r = sample_range(ctx, g, model, seed, id_base + lo, hi - lo, id_base, false);
   st->edges_examined += r.edges;
   st->spilled_samples += r.spilled;
   st->sample_launches += r.launches;
@@ -108,13 +109,24 @@ void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 // resumed when its ids are needed, or cancelled when they are not.  Sample
 // ids are fixed labels, so a speculative set is exactly the set the next
 // round needs and results are unchanged.
+//
+// Source elimination (R22, elim = true): sets are the non-empty root-less
+// sets in sample-id order; a round launches enough ids for the sets still
+// needed (from the kept fraction so far), keeps the first of them and
+// continues from the id after the last kept one.
 class RoundSampler {
  public:
-  RoundSampler(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, eim_stats* st)
-      : ctx_(ctx), g_(g), model_(model), seed_(seed), st_(st) {
+  RoundSampler(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, eim_stats* st, bool elim)
+      : ctx_(ctx), g_(g), model_(model), seed_(seed), st_(st), elim_(elim) {
     // opt-in (EIM_SPECULATE=1): measured on C2 the speculative round slows the
     // current round's critical chains as much as it fills their idle SMs
-    speculate_ = ctx->world == 1 && std::getenv("EIM_SPECULATE") != nullptr;
+    speculate_ = ctx->world == 1 && !elim && std::getenv("EIM_SPECULATE") != nullptr;
+  }
+
+  // Continue with an empty arena from sample id `id_base` (fresh final phase, R23).
+  void restart(uint64_t id_base) {
+    cancel();
+    id_base_ = next_id_ = id_base;
   }
   ~RoundSampler() {
     ex_.counts.release();
@@ -126,25 +138,32 @@ class RoundSampler {
   void grow(uint64_t& R, uint64_t to, uint64_t next_to) {
     if (to <= R) return;
     const auto t0 = clk::now();
+    if (elim_) {
+      grow_elim(R, to);
+      st_->ms_sample += ms_since(t0);
+      return;
+    }
+    st_->ids_sampled += to - R;
     if (ctx_->world > 1) {
-      sample_round(ctx_, g_, model_, seed_, R, to, st_, ex_);
+      sample_round(ctx_, g_, model_, seed_, id_base_, R, to, st_, ex_);
       R = to;
       return;
     }
     Round* cur = nullptr;
-    if (spec_ && spec_->first == R) {
+    if (spec_ && spec_->first == id_base_ + R) {
       cur = spec_;
       spec_ = nullptr;
       round_resume(ctx_, g_, *cur, stream_of(*cur));
     } else {
       cancel();
       cur = &ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, *cur, stream_of(*cur), false);
+      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, *cur, stream_of(*cur), false);
     }
     const uint64_t cur_end = R + cur->count;
     if (speculate_ && next_to > cur_end) {
       Round& nx = (cur == &ctx_->rounds[0]) ? ctx_->rounds[1] : ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, cur_end, next_to - cur_end, 0, true, nx, stream_of(nx), true);
+      round_launch(ctx_, g_, model_, seed_, id_base_ + cur_end, next_to - cur_end, id_base_, true, nx, stream_of(nx),
+                   true);
       spec_ = &nx;
     }
     const uint64_t use = std::min<uint64_t>(cur->count, to - R);
@@ -153,7 +172,7 @@ class RoundSampler {
     if (to > R) {  // the speculative range was shorter than needed: sample the rest now
       cancel();
       Round& rd = ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, R, to - R, 0, true, rd, stream_of(rd), false);
+      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, rd, stream_of(rd), false);
       account(round_finalize(ctx_, g_, rd, to - R));
       R = to;
     }
@@ -176,11 +195,36 @@ class RoundSampler {
     st_->sample_launches += r.launches;
     st_->ms_sample_kernel += r.kernel_ms;
   }
+  void grow_elim(uint64_t& R, uint64_t to) {
+    while (R < to) {
+      const uint64_t need = to - R;
+      // kept fraction so far (first launch: 1/4), 5% + 64 ids of slack
+      const double q = consumed_ ? std::max(1e-6, (double)std::max<uint64_t>(kept_, 1) / (double)consumed_) : 0.25;
+      const double want = std::ceil((double)need / q * 1.05) + 64.0;
+      const uint64_t count = (uint64_t)std::min(want, (double)(1ull << 29));
+      if (next_id_ + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids exhausted (< 2^62)");
+      Round& rd = ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, next_id_, count, next_id_ - R, true, rd, stream_of(rd), false,
+                   RF_DROP_ROOT | RF_DROP_EMPTY);
+      const SampleResult r = round_finalize(ctx_, g_, rd, need);
+      account(r);
+      R += r.kept;
+      next_id_ += r.consumed;
+      kept_ += r.kept;
+      consumed_ += r.consumed;
+      st_->ids_sampled += r.consumed;
+    }
+  }
+
   eim_ctx* ctx_;
   const eim_graph* g_;
   eim_model model_;
   uint64_t seed_;
   eim_stats* st_;
+  bool elim_;
+  uint64_t id_base_ = 0;              // sample id of set index 0 (plain runs)
+  uint64_t next_id_ = 0;              // next sample id (source elimination)
+  uint64_t kept_ = 0, consumed_ = 0;  // kept sets / ids used so far (source elimination)
   Exchange ex_;
   bool speculate_ = false;
   Round* spec_ = nullptr;
@@ -189,9 +233,14 @@ class RoundSampler {
 }  // namespace
 
 void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
-             uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, eim_stats* st) {
+             uint64_t seed, uint32_t flags, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
+             eim_stats* st) {
   const auto t_start = clk::now();
   const uint32_t n = g->view.n;
+  const bool elim = (flags & EIM_F_SOURCE_ELIM) != 0, fresh = (flags & EIM_F_FRESH_FINAL) != 0;
+  if (elim && ctx->world > 1) fail(EIM_E_INVAL, "EIM_F_SOURCE_ELIM needs a single-GPU context");
+  if (elim && !graph_has_proper_edge(ctx, g))
+    fail(EIM_E_INVAL, "EIM_F_SOURCE_ELIM: the graph has no edge u->v with u != v (every set would be empty)");
   eim_imm_params_t p;
   imm_params(n, k, eps, ell, &p);
   std::memset(st, 0, sizeof(*st));
@@ -199,11 +248,12 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   st->lambda_s = p.lambda_s;
   const uint64_t launches0 = ctx->kernel_launches;
   cudaStream_t s = ctx->stream;
-  // fresh arena + coverage for this graph
-  arena_reset(ctx);
+  // fresh arena + coverage for this graph; R is log-encoded with the graph (NEXT-2)
+  const uint32_t arena_b = g->packed ? bit_width((uint64_t)n - 1) : 32u;
+  arena_reset(ctx, arena_b);
   ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
   EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
-  RoundSampler sampler(ctx, g, model, seed, st);
+  RoundSampler sampler(ctx, g, model, seed, st, elim);
   std::vector<uint32_t> S(k);
   uint64_t R = 0, cov = 0;
   uint64_t R_selected = UINT64_MAX;  // |R| the last NodeSelection ran on
@@ -229,6 +279,13 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
     }
     st->lb = LB;
     const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
+    if (fresh) {  // R23: the final sets are drawn afresh from ids 2^61..
+      sampler.restart(EIM_FRESH_BASE);
+      arena_reset(ctx, arena_b);
+      EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
+      R = 0;
+      R_selected = UINT64_MAX;
+    }
     sampler.grow(R, theta, 0);
     sampler.cancel();
   } catch (...) {
@@ -244,6 +301,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   st->theta = R;
   st->cov = cov;
   st->arena_elems = arena_cursor(ctx);
+  st->arena_bytes = ctx->arena_b == 32 ? 4 * st->arena_elems : 4 * arena_words(st->arena_elems, ctx->arena_b);
   if (theta_out) *theta_out = R;
   if (spread_out) *spread_out = (double)n * (double)cov / (double)R;
   st->kernel_launches = ctx->kernel_launches - launches0;

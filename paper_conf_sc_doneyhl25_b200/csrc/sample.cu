@@ -34,7 +34,7 @@
 #include <cstdlib>
 #include <string>
 
-#include "eim_internal.h"
+#include "arena_view.cuh"
 #include "philox.cuh"
 
 namespace eim {
@@ -249,11 +249,11 @@ __device__ __forceinline__ void task_push1(const RoundView& R, SampleCtl* ctl, u
 // visit v for the traversal of sub-group o (sample s_local, ring head `head`):
 // table insert; a new member is appended to o's ring with its row (loaded
 // alongside the insert), or becomes a one-vertex task when the ring is full.
-template <int G>
-__device__ __forceinline__ void visit_for(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+template <int G, class GV>
+__device__ __forceinline__ void visit_for(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                           uint32_t s_local, uint32_t head, uint32_t W, uint32_t v) {
-  const unsigned long long e0 = g.off[v], e1 = g.off[v + 1];
-  const uint32_t T = g.thr[v];
+  const unsigned long long e0 = g_off(g, v), e1 = g_off(g, v + 1);
+  const uint32_t T = g_thr(g, v, e1 - e0);
   const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
   if (ins > 0) {
     const uint32_t pos = atomicAdd(&o.gc->tail, 1u);
@@ -326,8 +326,8 @@ __device__ __forceinline__ uint32_t min4(const uint4& w) { return min(min(w.x, w
 // e = 4q + i; it belongs to c's row unless the quad is the row's first
 // (i < wlo) or last (i > whi) and straddles a neighbour row.  A live edge is
 // parked in o's live list (visited directly when the list is full).
-template <int G>
-__device__ __forceinline__ void park_live(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+template <int G, class GV>
+__device__ __forceinline__ void park_live(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                        const Cur& c, uint4 w, uint32_t s_local, uint32_t head, uint32_t W) {
   const GroupRows<G>& rw = *o.rw;
   uint32_t live = (w.x <= c.T ? 1u : 0u) | (w.y <= c.T ? 2u : 0u) | (w.z <= c.T ? 4u : 0u) | (w.w <= c.T ? 8u : 0u);
@@ -340,7 +340,7 @@ __device__ __forceinline__ void park_live(const GraphView& g, const RoundView& R
     const unsigned long long e = (q << 2) + i;
     const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
     if (p < LIVE_CAP) o.live_e[p] = e;
-    else visit_for<G>(g, R, ctl, o, s_local, head, W, g.nbr[e]);
+    else visit_for<G>(g, R, ctl, o, s_local, head, W, g_nbr(g, e));
   }
 }
 
@@ -354,8 +354,8 @@ __device__ __forceinline__ void park_live(const GraphView& g, const RoundView& R
 #ifndef EIM_SWEEP_U
 #define EIM_SWEEP_U 2
 #endif
-template <int G, int NT, bool HOIST, int U>
-__device__ __forceinline__ void sweep_runs(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+template <int G, int NT, bool HOIST, int U, class GV>
+__device__ __forceinline__ void sweep_runs(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                            uint32_t nrows, uint32_t lo, uint32_t hi, int t, uint32_t c2, uint32_t c3,
                                            const EdgeConsts& E, uint32_t s_local, uint32_t head, uint32_t W) {
   const GroupRows<G>& rw = *o.rw;
@@ -387,8 +387,8 @@ __device__ __forceinline__ void sweep_runs(const GraphView& g, const RoundView& 
   }
 }
 
-template <int G, int NT>
-__device__ __forceinline__ void sweep_any(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+template <int G, int NT, class GV>
+__device__ __forceinline__ void sweep_any(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                           uint32_t nrows, uint32_t lo, uint32_t hi, int t, uint64_t s,
                                           uint32_t s_local, uint32_t head, uint32_t W, bool hoist) {
   const uint32_t c2 = (uint32_t)s, c3 = ctr_hi(s, TAG_EDGE);
@@ -399,8 +399,8 @@ __device__ __forceinline__ void sweep_any(const GraphView& g, const RoundView& R
 
 // A warp claims and sweeps chunks of o's current job until none is left.
 // Returns true if it swept anything.
-template <int G>
-__device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
+template <int G, class GV>
+__device__ __forceinline__ bool work_job(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                          int lane, uint32_t W) {
   Job& j = o.gc->job;
   bool any = false;
@@ -428,8 +428,8 @@ __device__ __forceinline__ bool work_job(const GraphView& g, const RoundView& R,
 }
 
 // Warp-level: join the open jobs of the other sub-groups of the block.
-template <int G, int NSG>
-__device__ __forceinline__ bool help_others(const GraphView& g, const RoundView& R, SampleCtl* ctl,
+template <int G, int NSG, class GV>
+__device__ __forceinline__ bool help_others(const GV& g, const RoundView& R, SampleCtl* ctl,
                                             unsigned char* smem, int gi, int lane, uint32_t W) {
   bool any = false;
   if (NSG < 2) return false;
@@ -477,8 +477,8 @@ __device__ __forceinline__ uint32_t stage_row(GroupRows<G>& rw, int gtid, unsign
 // the traversals is the unique reachable set of the sampled world, whatever
 // the split.  Returns 0, FLAG_TABLE or FLAG_CANCEL; found = new members
 // inserted by this traversal.
-template <int G, int NSG>
-__device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView& R, SampleCtl* ctl,
+template <int G, int NSG, class GV>
+__device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, SampleCtl* ctl,
                                              unsigned char* smem, int gi, uint32_t s_local, bool root,
                                              unsigned long long poff, uint32_t nseed, uint32_t W, int gtid,
                                              uint32_t& found, uint32_t spill_quads, uint32_t task_quads,
@@ -526,11 +526,11 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
     // pool lines may be cached from a neighbouring task: read through L2
     for (uint32_t t = gtid; t < nseed; t += G) {
       const uint32_t v = __ldcg(R.pool + poff + t);
-      const unsigned long long e0 = g.off[v];
+      const unsigned long long e0 = g_off(g, v), e1 = g_off(g, v + 1);
       me.ring[t] = v;
       me.rr.e0[t] = e0;
-      me.rr.d[t] = (uint32_t)(g.off[v + 1] - e0);
-      me.rr.T[t] = g.thr[v];
+      me.rr.d[t] = (uint32_t)(e1 - e0);
+      me.rr.T[t] = g_thr(g, v, e1 - e0);
     }
   }
   gsync<G>(gi);
@@ -671,7 +671,7 @@ __device__ __forceinline__ uint32_t traverse(const GraphView& g, const RoundView
     mark(1);
     // ---- visit the parked live neighbours, one per thread
     const uint32_t nl = min(*(volatile uint32_t*)&gc.nlive, LIVE_CAP);
-    for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, g.nbr[me.live_e[t]]);
+    for (uint32_t t = gtid; t < nl; t += G) visit_for<G>(g, R, ctl, me, s_local, head, W, g_nbr(g, me.live_e[t]));
     swept += total;
     nbatch++;
     nquads += total;
@@ -737,8 +737,8 @@ constexpr int ic_min_blocks() {
   return EIM_IC_THREADS_SM / (G * NSG) > 0 ? EIM_IC_THREADS_SM / (G * NSG) : 1;
 }
 
-template <int G, int NSG>
-__global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GraphView g, RoundView R, uint64_t count, uint32_t W,
+template <int G, int NSG, class GV>
+__global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV g, RoundView R, uint64_t count, uint32_t W,
                                                       SampleCtl* ctl, uint32_t spill_quads, uint32_t task_quads,
                                                       uint32_t help_min) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -802,7 +802,8 @@ size_t ic_smem(uint32_t W) {
 // floor(tau * d / 2^32) of u's row (the prefix-scan choice under WC
 // weights); the walk stops when d^-(u) = 0 or the chosen vertex is already in
 // the set.  One thread per walk; visited set = the round table.
-__global__ void __launch_bounds__(256) lt_kernel(GraphView g, RoundView R, uint64_t count, SampleCtl* ctl) {
+template <class GV>
+__global__ void __launch_bounds__(256) lt_kernel(GV g, RoundView R, uint64_t count, SampleCtl* ctl) {
   const PhiloxKey& K = R.K;
   unsigned long long edges_acc = 0;
   for (;;) {
@@ -817,13 +818,13 @@ __global__ void __launch_bounds__(256) lt_kernel(GraphView g, RoundView R, uint6
     uint32_t L = 1;
     unsigned long long steps = 0;
     while (ok) {
-      const unsigned long long e0 = g.off[u], e1 = g.off[u + 1];
+      const unsigned long long e0 = g_off(g, u), e1 = g_off(g, u + 1);
       if (e1 == e0) break;
       ++steps;
       const uint4 w = philox_at((uint64_t)(u >> 2), s, TAG_LT, K);
       const uint32_t tau = word_of(w, u & 3u);
       const unsigned long long j = __umul64hi((unsigned long long)tau << 32, e1 - e0);
-      const uint32_t v = g.nbr[e0 + j];
+      const uint32_t v = g_nbr(g, e0 + j);
       const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
       if (ins == 0) break;
       if (ins < 0) ok = false;
@@ -859,13 +860,57 @@ __global__ void place_sets_kernel(const uint64_t* __restrict__ excl, const uint3
   }
 }
 
+// Source-vertex elimination (R22).  roots[i] = root of sample
+// first+i (Alg. 2 l.6, the same draw the traversal started from).
+__global__ void roots_kernel(uint64_t first, uint64_t count, uint32_t n, PhiloxKey K, uint32_t* __restrict__ roots) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride)
+    roots[i] = draw_root(first + i, n, K);
+}
+
+// sizes[i] -= 1 (the root leaves the set); keep[i] = set non-empty.
+__global__ void drop_root_sizes_kernel(uint32_t* __restrict__ sizes, uint64_t count, uint32_t* __restrict__ keep) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= count; i += stride) {
+    if (i == count) {
+      if (keep) keep[i] = 0;
+      continue;
+    }
+    const uint32_t z = sizes[i] - 1u;
+    sizes[i] = z;
+    if (keep) keep[i] = z != 0u;
+  }
+}
+
+// kidx = exclusive scan of keep.  The need-th kept sample (kidx[i] ==
+// need-1, kept) ends the ids taken: *consumed = i + 1.
+__global__ void find_consumed_kernel(const uint32_t* __restrict__ kidx, uint64_t count, uint32_t need,
+                                     unsigned long long* __restrict__ consumed) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride)
+    if (kidx[i] == need - 1u && kidx[i + 1] == need) *consumed = i + 1;
+}
+
+// Kept sets, compacted: ksizes[kidx[i]] = sizes[i] for the kept i < consumed.
+__global__ void compact_sizes_kernel(const uint32_t* __restrict__ sizes, const uint32_t* __restrict__ kidx,
+                                     uint64_t consumed, uint32_t* __restrict__ ksizes) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < consumed; i += stride)
+    if (kidx[i + 1] != kidx[i]) ksizes[kidx[i]] = sizes[i];
+}
+
 // Every live table entry is a member: arena[start(s) + fill[s]++] = v.
 // IC (off != nullptr): the in-edges examined by a set are exactly the
 // in-edges of its members (each member is expanded once), summed into *esum.
+// With roots (source elimination) the root entry of a sample is not stored
+// (its edges still count: the traversal examined them) and, with kidx, the
+// set index of sample s is set_index0 + kidx[s] (empty sets dropped).
+template <class GV>
 __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint64_t nslots,
                                const uint64_t* __restrict__ set_start, uint64_t set_index0, uint32_t use,
-                               uint32_t* __restrict__ fill, uint32_t* __restrict__ arena, uint32_t* __restrict__ C,
-                               const uint64_t* __restrict__ off, unsigned long long* __restrict__ esum) {
+                               uint32_t* __restrict__ fill, uint32_t* __restrict__ arena, uint32_t ab,
+                               uint32_t* __restrict__ C, GV g, bool ic, unsigned long long* __restrict__ esum,
+                               const uint32_t* __restrict__ roots, const uint32_t* __restrict__ kidx) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   unsigned long long e = 0;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nslots; i += stride) {
@@ -874,12 +919,14 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
     const uint32_t s_local = (uint32_t)(k >> 32) - 1u;
     if (s_local >= use) continue;  // speculative samples beyond the ones kept
     const uint32_t v = (uint32_t)k;
+    if (ic) e += g_off(g, v + 1) - g_off(g, v);
+    if (roots && v == roots[s_local]) continue;
+    const uint64_t si = set_index0 + (kidx ? kidx[s_local] : s_local);
     const uint32_t p = atomicAdd(&fill[s_local], 1u);
-    arena[set_start[set_index0 + s_local] + p] = v;
+    arena_put(arena, set_start[si] + p, ab, v);
     if (C) atomicAdd(&C[v], 1u);
-    if (off) e += off[v + 1] - off[v];
   }
-  if (off) {
+  if (ic) {
     for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(FULL, e, o);
     if ((threadIdx.x & 31) == 0 && e) atomicAdd(esum, e);
   }
@@ -927,8 +974,10 @@ constexpr uint32_t IC_W = 1024;  // shared-memory frontier ring per group
 }  // namespace
 
 // ------------------------------------------------------------------ host
-void arena_reset(eim_ctx* ctx) {
+void arena_reset(eim_ctx* ctx, uint32_t b) {
+  ctx->arena_b = b;
   ctx->arena.reserve(sizeof(uint32_t) * (1u << 22), false, ctx->stream);
+  if (b < 32) EIM_CUDA(cudaMemsetAsync(ctx->arena.p, 0, ctx->arena.bytes, ctx->stream));
   ctx->ctl.reserve(sizeof(SampleCtl) + 2 * sizeof(unsigned long long), false, ctx->stream);
   EIM_CUDA(cudaMemsetAsync(ctx->ctl.p, 0, sizeof(SampleCtl) + 2 * sizeof(unsigned long long), ctx->stream));
   ctx->est_mean_size = 0;
@@ -937,13 +986,26 @@ void arena_reset(eim_ctx* ctx) {
 
 uint64_t arena_cursor(eim_ctx* ctx) { return ctx->arena_used; }
 
+void arena_ensure(eim_ctx* ctx, uint64_t elems) {
+  const uint32_t b = ctx->arena_b;
+  const size_t before = ctx->arena.bytes;
+  ctx->arena.reserve(std::max<uint64_t>(arena_words(elems, b), 1) * sizeof(uint32_t), true, ctx->stream);
+  // encoded: containers past the last used bit stay zero (writers OR into them)
+  if (b < 32 && ctx->arena.bytes > before) {
+    const uint64_t used = (ctx->arena_used * b + 31) / 32;
+    EIM_CUDA(cudaMemsetAsync(ctx->arena.as<uint32_t>() + used, 0, ctx->arena.bytes - used * sizeof(uint32_t),
+                             ctx->stream));
+  }
+}
+
 void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
   ctx->set_start.reserve(num_sets * sizeof(uint64_t), true, ctx->stream);
   ctx->set_len.reserve(num_sets * sizeof(uint32_t), true, ctx->stream);
 }
 
 void round_release(Round& rd) {
-  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.edges, &rd.fill, &rd.excl, &rd.ctl, &rd.queue, &rd.dbg};
+  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.edges, &rd.fill, &rd.excl, &rd.ctl, &rd.queue, &rd.dbg,
+                 &rd.roots, &rd.kidx, &rd.ksizes};
   for (DevBuf* x : b) x->release();
   for (cudaEvent_t& e : rd.ev) {
     if (e) cudaEventDestroy(e);
@@ -971,22 +1033,29 @@ static uint32_t ring_w() {
 
 static uint32_t help_min() { return env_u32("EIM_HELP_QUADS", 1024); }
 
-template <int G, int NSG>
-static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint64_t count, SampleCtl* ctl,
-                      cudaStream_t st, bool spare_sm_slot) {
-  const uint32_t W = ring_w();
-  const size_t smem = ic_smem<G, NSG>(W);
-  auto kern = ic_kernel<G, NSG>;
+template <int G, int NSG, class K, class GV>
+static void launch_ic_on(eim_ctx* ctx, K kern, const GV& gv, const RoundView& R, uint64_t count, SampleCtl* ctl,
+                         cudaStream_t st, bool spare_sm_slot, uint32_t W, size_t smem) {
   EIM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, G * NSG, smem));
   if (per_sm < 1) fail(EIM_E_CUDA, "sampler does not fit on an SM");
   if (spare_sm_slot && per_sm > 1) per_sm -= 1;
   const uint64_t blocks = std::max<uint64_t>(1, (uint64_t)per_sm * ctx->sm_count);
-  kern<<<(uint32_t)blocks, G * NSG, smem, st>>>(g->view, R, count, W, ctl, spill_quads(), task_quads(), help_min());
+  kern<<<(uint32_t)blocks, G * NSG, smem, st>>>(gv, R, count, W, ctl, spill_quads(), task_quads(), help_min());
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
 }
+
+template <int G, int NSG>
+static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint64_t count, SampleCtl* ctl,
+                      cudaStream_t st, bool spare_sm_slot) {
+  const uint32_t W = ring_w();
+  const size_t smem = ic_smem<G, NSG>(W);
+  if (g->packed) launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, PackedGraphView>, g->pview, R, count, ctl, st, spare_sm_slot, W, smem);
+  else launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, GraphView>, g->view, R, count, ctl, st, spare_sm_slot, W, smem);
+}
+
 
 static RoundView round_view(Round& rd) {
   return RoundView{rd.table.as<unsigned long long>(),
@@ -1014,10 +1083,12 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
     launch_ic<IC_G, IC_NSG>(ctx, g, R, rd.count, ctl, st, spare_sm_slot);
   } else {
     int per_sm = 0;
-    EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel, 256, 0));
+    EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lt_kernel<GraphView>, 256, 0));
     if (spare_sm_slot && per_sm > 1) per_sm -= 1;
     uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
-    lt_kernel<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(g->view, R, rd.count, ctl);
+    const uint32_t grid = (uint32_t)std::max<uint64_t>(blocks, 1);
+    if (g->packed) lt_kernel<<<grid, 256, 0, st>>>(g->pview, R, rd.count, ctl);
+    else lt_kernel<<<grid, 256, 0, st>>>(g->view, R, rd.count, ctl);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
   }
@@ -1077,8 +1148,10 @@ void round_resume(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st) 
 }
 
 void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t first,
-                  uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot) {
+                  uint64_t count, uint64_t set_base, bool hist, Round& rd, cudaStream_t st, bool spare_sm_slot,
+                  uint32_t rflags) {
   if (count == 0) return;
+  rd.rflags = rflags;
   if (count >= 0x3FFFFFF0ull) fail(EIM_E_INVAL, "at most 2^30 sets per sampler launch");
   if (!rd.ev[0])
     for (cudaEvent_t& e : rd.ev) EIM_CUDA(cudaEventCreate(&e));
@@ -1096,7 +1169,8 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   // table capacity: >= 4x the expected members (mean set size of earlier
   // rounds, else 64), at least 2^20 slots
   const double mean = ctx->est_mean_size > 0 ? ctx->est_mean_size : 64.0;
-  uint32_t bits = 20;
+  // EIM_TABLE_BITS: smallest table (tests force overflow and the redo path)
+  uint32_t bits = std::min<uint32_t>(std::max<uint32_t>(env_u32("EIM_TABLE_BITS", 20), 4), 31);
   while (bits < 31 && (double)(1ull << bits) < 4.0 * mean * (double)count) bits++;
   rd.bits = bits;
   round_start(ctx, g, rd, st, spare_sm_slot);
@@ -1167,50 +1241,109 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     break;
   }
   rd.launched = false;
+  res.kept = res.consumed = use;
   if (use == 0) return res;
+  const bool drop_root = (rd.rflags & RF_DROP_ROOT) != 0;
+  const bool drop_empty = drop_root && (rd.rflags & RF_DROP_EMPTY) != 0;
+  uint32_t* sizes = rd.sizes.as<uint32_t>();
+  uint32_t* roots = nullptr;
+  uint32_t* kidx = nullptr;
+  uint64_t consumed = use, nsets = use;
+  size_t tmp = 0, tmp2 = 0;
+  if (drop_root) {
+    // ---- source elimination (R22): roots out of the sets; with drop_empty
+    // only the first `use` non-empty sets are kept and the ids up to the
+    // last kept one are consumed.
+    const uint64_t span = drop_empty ? rd.count : use;
+    rd.roots.reserve(span * sizeof(uint32_t), false, st);
+    roots = rd.roots.as<uint32_t>();
+    roots_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(rd.first, span, g->view.n, philox_key(rd.seed), roots);
+    EIM_CUDA(cudaGetLastError());
+    if (drop_empty) {
+      rd.kidx.reserve((span + 1) * sizeof(uint32_t), false, st);
+      rd.ksizes.reserve(span * sizeof(uint32_t), false, st);
+      kidx = rd.kidx.as<uint32_t>();
+    }
+    drop_root_sizes_kernel<<<grid_for(ctx, span + 1, 256), 256, 0, st>>>(sizes, span, kidx);
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches += 2;
+    if (drop_empty) {
+      EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, kidx, kidx, span + 1, st));
+      ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+      EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, kidx, kidx, span + 1, st));
+      uint32_t* h32 = reinterpret_cast<uint32_t*>(&h->consumed);
+      EIM_CUDA(cudaMemcpyAsync(h32, kidx + span, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+      EIM_CUDA(cudaStreamSynchronize(st));
+      const uint64_t kept_total = *h32;
+      consumed = span;
+      nsets = kept_total;
+      if (kept_total >= use) {
+        nsets = use;
+        find_consumed_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(kidx, span, (uint32_t)use, &ctl->consumed);
+        EIM_CUDA(cudaGetLastError());
+        EIM_CUDA(cudaMemcpyAsync(&h->consumed, &ctl->consumed, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        EIM_CUDA(cudaStreamSynchronize(st));
+        consumed = h->consumed;
+        ctx->kernel_launches += 1;
+      }
+      if (nsets)
+        compact_sizes_kernel<<<grid_for(ctx, consumed, 256), 256, 0, st>>>(sizes, kidx, consumed,
+                                                                          rd.ksizes.as<uint32_t>());
+      EIM_CUDA(cudaGetLastError());
+      ctx->kernel_launches += 2;
+      sizes = rd.ksizes.as<uint32_t>();
+    }
+  }
+  res.kept = nsets;
+  res.consumed = consumed;
   // ---- sizes -> offsets (sample-id order) -> arena placement -> scatter + histogram
   uint64_t* excl = rd.excl.as<uint64_t>();
-  ensure_sets(ctx, rd.first + use - rd.set_base);
-  sizes_to_offsets_kernel<<<grid_for(ctx, use + 1, 256), 256, 0, st>>>(rd.sizes.as<uint32_t>(), use, excl);
+  const uint64_t set_index0 = rd.first - rd.set_base;
+  ensure_sets(ctx, set_index0 + std::max<uint64_t>(nsets, 1));
+  sizes_to_offsets_kernel<<<grid_for(ctx, nsets + 1, 256), 256, 0, st>>>(sizes, nsets, excl);
   EIM_CUDA(cudaGetLastError());
-  size_t tmp = 0, tmp2 = 0;
   const bool ic = rd.model == EIM_IC;
   unsigned long long* d_edges_sum = &ctl->edges;  // IC: summed by the scatter; LT: reduced from per-walk steps
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, use + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, nsets + 1, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, consumed, st));
   ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, use + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, use, st));
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, nsets + 1, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, consumed, st));
   else EIM_CUDA(cudaMemsetAsync(d_edges_sum, 0, sizeof(unsigned long long), st));
-  EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + use, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + nsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   const uint64_t total = h->ticket, cursor = ctx->arena_used;
-  ctx->arena.reserve((cursor + total) * sizeof(uint32_t), true, st);
-  const uint64_t set_index0 = rd.first - rd.set_base;
-  place_sets_kernel<<<grid_for(ctx, use, 256), 256, 0, st>>>(excl, rd.sizes.as<uint32_t>(), use, cursor, set_index0,
-                                                              ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
-  EIM_CUDA(cudaGetLastError());
-  EIM_CUDA(cudaMemsetAsync(rd.fill.p, 0, use * sizeof(uint32_t), st));
+  arena_ensure(ctx, cursor + total);
+  if (nsets) {
+    place_sets_kernel<<<grid_for(ctx, nsets, 256), 256, 0, st>>>(excl, sizes, nsets, cursor, set_index0,
+                                                                  ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
+    EIM_CUDA(cudaGetLastError());
+  }
+  EIM_CUDA(cudaMemsetAsync(rd.fill.p, 0, consumed * sizeof(uint32_t), st));
   const uint64_t nslots = 1ull << rd.bits;
-  scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
-      rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
-      (uint32_t)use, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(),
-      rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, ic ? g->view.off : nullptr, d_edges_sum);
+  auto scatter = [&](auto gv) {
+    scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
+        rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
+        (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
+        rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_sum, roots, kidx);
+  };
+  if (g->packed) scatter(g->pview);
+  else scatter(g->view);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;
   ctx->arena_used = cursor + total;
   EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   res.edges = h->edges;
-  ctx->est_mean_size = std::max(1.0, (double)total / (double)use);
+  ctx->est_mean_size = std::max(1.0, (double)(total + (drop_root ? consumed : 0)) / (double)consumed);
   return res;
 }
 
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
-                          uint64_t first, uint64_t count, uint64_t set_base, bool hist) {
+                          uint64_t first, uint64_t count, uint64_t set_base, bool hist, uint32_t rflags) {
   if (count == 0) return SampleResult{};
   Round& rd = ctx->rounds[0];
-  round_launch(ctx, g, model, seed, first, count, set_base, hist, rd, ctx->stream, false);
+  round_launch(ctx, g, model, seed, first, count, set_base, hist, rd, ctx->stream, false, rflags);
   return round_finalize(ctx, g, rd, count);
 }
 

@@ -24,7 +24,7 @@
 
 #include <cub/cub.cuh>
 
-#include "eim_internal.h"
+#include "arena_view.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -69,11 +69,11 @@ __global__ void compact_kernel(const uint32_t* __restrict__ C, const uint32_t* _
   }
 }
 
-__global__ void remap_kernel(const uint32_t* __restrict__ arena, uint64_t total, const uint32_t* __restrict__ cidx,
-                             uint32_t* __restrict__ arena_c) {
+__global__ void remap_kernel(const uint32_t* __restrict__ arena, uint32_t ab, uint64_t total,
+                             const uint32_t* __restrict__ cidx, uint32_t* __restrict__ arena_c) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride)
-    arena_c[i] = cidx[arena[i]];
+    arena_c[i] = cidx[arena_get(arena, i, ab)];
 }
 
 // inverted index fill: one warp per set.  off[x] holds the END of x's list
@@ -263,8 +263,8 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
   // ---- 2. arena in candidate indices + inverted index
   ctx->arena_c.reserve(std::max<uint64_t>(total, 1) * 4, false, st);
   if (total)
-    remap_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(ctx->arena.as<uint32_t>(), total, ctx->cidx.as<uint32_t>(),
-                                                              ctx->arena_c.as<uint32_t>());
+    remap_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(ctx->arena.as<uint32_t>(), ctx->arena_b, total,
+                                                              ctx->cidx.as<uint32_t>(), ctx->arena_c.as<uint32_t>());
   EIM_CUDA(cub::DeviceScan::InclusiveSum(ctx->scratch.p, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
   ctx->inv.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
   if (num_sets > 0 && total > 0) {

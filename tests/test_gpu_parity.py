@@ -234,3 +234,146 @@ def test_C3_sampled_sets_and_imm(eim, ctx, graphs):
         _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
     finally:
         eim.eim_graph_free(g)
+
+
+# ---------------------------------------------------------------- NEXT rows
+# NEXT-1 source elimination (R22), NEXT-4 fresh final phase (R23): same bar.
+ELIM, FRESH = oracle.SOURCE_ELIM, oracle.FRESH_FINAL
+assert (ELIM, FRESH) == (1, 2)  # == EIM_F_SOURCE_ELIM, EIM_F_FRESH_FINAL
+
+
+def _imm_equal_flags(eim, ctx, g, off, nbr, k, eps, ell, model, seed, flags):
+    seeds, theta, spread, st = eim.eim_imm_run(ctx, g, k, eps, ell, model, seed, flags=flags)
+    ref = oracle.imm(off, nbr, k, eps, ell, model, seed, nthreads=NT, flags=flags)
+    assert np.array_equal(seeds, ref["seeds"]), (model, seed, flags)
+    for key in ("theta_i", "cov_i", "lb", "cov", "edges_examined", "arena_elems", "ids_sampled"):
+        assert st[key] == ref[key], (key, st[key], ref[key])
+    assert theta == ref["theta"] and spread == ref["spread"]
+    return st
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_sample_rrr_source_elim(eim, ctx, graphs, model, spill_mode):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        for first, count in ((0, 20000), (2**45 + 5, 301), (oracle.FRESH_BASE, 999)):
+            go, gm = eim.eim_sample_rrr(ctx, g, model, 6, first, count, flags=ELIM)
+            ro, rm, _ = oracle.sample(off, nbr, model, 6, first, count, nthreads=NT, flags=ELIM)
+            assert np.array_equal(go, ro) and np.array_equal(gm, rm), (first, count)
+            assert eim.eim_get_stats(ctx)["edges_examined"] == oracle.sample(
+                off, nbr, model, 6, first, count, nthreads=NT)[2]
+    finally:
+        eim.eim_graph_free(g)
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+@pytest.mark.parametrize("flags", [ELIM, FRESH, ELIM | FRESH])
+def test_imm_flags_C1(eim, ctx, graphs, model, flags):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        for seed in (1, 2, 3):
+            for k, eps in ((5, 0.5), (50, 0.2), (1024, 0.5)):
+                _imm_equal_flags(eim, ctx, g, off, nbr, k, eps, 1.0, model, seed, flags)
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_imm_flags_special_graphs(eim, ctx):
+    for off, nbr in (inputs.path_graph(32), inputs.cycle_graph(700), inputs.star_out(90),
+                     inputs.from_edges(6, [(0, 0), (4, 5)])):
+        g = eim.eim_load_graph_csr(ctx, off, nbr)
+        try:
+            for model in ("IC", "LT"):
+                for flags in (ELIM, FRESH | ELIM):
+                    _imm_equal_flags(eim, ctx, g, off, nbr, 3, 0.5, 1.0, model, 7, flags)
+        finally:
+            eim.eim_graph_free(g)
+    for off, nbr in (inputs.empty_graph(64), inputs.from_edges(4, [(0, 0), (2, 2)])):
+        g = eim.eim_load_graph_csr(ctx, off, nbr)
+        try:
+            with pytest.raises(eim.EimError) as ei:
+                eim.eim_imm_run(ctx, g, 1, 0.5, 1.0, "IC", 1, flags=ELIM)
+            assert ei.value.status == eim.EIM_E_INVAL
+            _imm_equal_flags(eim, ctx, g, off, nbr, 2, 0.5, 1.0, "IC", 1, FRESH)
+        finally:
+            eim.eim_graph_free(g)
+
+
+@pytest.mark.parametrize("flags", [ELIM, FRESH | ELIM])
+def test_C2_imm_flags(eim, ctx, graphs, flags):
+    c = inputs.CONFIGS["C2"]
+    off, nbr = graphs("C2")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        go, gm = eim.eim_sample_rrr(ctx, g, "IC", 1, 0, 2000, flags=ELIM)
+        ro, rm, _ = oracle.sample(off, nbr, "IC", 1, 0, 2000, nthreads=NT, flags=ELIM)
+        assert np.array_equal(go, ro) and np.array_equal(gm, rm)
+        st = _imm_equal_flags(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1, flags)
+        assert st["ids_sampled"] > st["theta"]
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_C3_imm_source_elim(eim, ctx, graphs):
+    c = inputs.CONFIGS["C3"]
+    off, nbr = graphs("C3")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        _imm_equal_flags(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1, ELIM)
+    finally:
+        eim.eim_graph_free(g)
+
+
+# NEXT-2: log-encoded graph store (R24).  Results must equal the plain store's
+# oracle outputs; the store's size must equal the containers R24 defines.
+LOGENC = 1  # EIM_G_LOG_ENCODE
+
+
+def _packed_bytes(off, nbr):
+    n, m = off.size - 1, nbr.size
+    boff = oracle.log_bits(m)
+    bnbr = oracle.log_bits(int(nbr.max()) if m else 0)
+    return 4 * ((((n + 1) * boff + 31) // 32 + 2) + ((m * bnbr + 31) // 32 + 2))
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_log_encoded_graph_C1(eim, ctx, graphs, model, spill_mode):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC)
+    try:
+        assert eim.eim_graph_bytes(g) == _packed_bytes(off, nbr)
+        _sets_equal(eim, ctx, g, off, nbr, model, 2, 0, 20000)
+        _sets_equal(eim, ctx, g, off, nbr, model, 2, 2**50 + 9, 500)
+        _imm_equal(eim, ctx, g, off, nbr, 20, 0.3, 1.0, model, 4)
+        _imm_equal_flags(eim, ctx, g, off, nbr, 5, 0.5, 1.0, model, 4, ELIM | FRESH)
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_log_encoded_special_graphs(eim, ctx):
+    for off, nbr in (inputs.empty_graph(64), inputs.path_graph(32), inputs.cycle_graph(3000), inputs.star_out(90),
+                     inputs.from_edges(3, [(0, 1), (0, 2)]), inputs.rmat(600, 60000, seed=4)):
+        g = eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC)
+        try:
+            assert eim.eim_graph_bytes(g) == _packed_bytes(off, nbr)
+            for model in ("IC", "LT"):
+                _sets_equal(eim, ctx, g, off, nbr, model, 9, 0, 700)
+                _imm_equal(eim, ctx, g, off, nbr, 3, 0.5, 1.0, model, 7)
+        finally:
+            eim.eim_graph_free(g)
+
+
+def test_log_encoded_C2_imm(eim, ctx, graphs):
+    c = inputs.CONFIGS["C2"]
+    off, nbr = graphs("C2")
+    g = eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC)
+    try:
+        packed = eim.eim_graph_bytes(g)
+        assert packed == _packed_bytes(off, nbr)
+        assert packed < 0.7 * (8 * off.size + 4 * nbr.size + 4 * (off.size - 1))
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 0, 2000)
+        _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
+    finally:
+        eim.eim_graph_free(g)
