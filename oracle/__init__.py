@@ -91,6 +91,11 @@ def _load():
             "orc_imm_params": (I32, [U32, U32, D, D, ctypes.POINTER(Params)]),
             "orc_imm": (I32, [U32, P, P, U32, D, D, I32, U64, I32, P, P, P, ctypes.POINTER(ImmStats)]),
             "orc_imm_ex": (I32, [U32, P, P, U32, D, D, I32, U64, U32, I32, P, P, P, ctypes.POINTER(ImmStats)]),
+            "orc_ic_live_w": (I32, [U32, U32]),
+            "orc_lt_choice_w": (U32, [U32, P, U64]),
+            "orc_lt_weights_ok": (I32, [U32, P, P]),
+            "orc_sample_w": (ctypes.POINTER(_Arena), [U32, P, P, P, I32, U64, U64, U64, U32, I32]),
+            "orc_imm_w": (I32, [U32, P, P, P, U32, D, D, I32, U64, U32, I32, P, P, P, ctypes.POINTER(ImmStats)]),
             "orc_log_bits": (U32, [U64]),
             "orc_log_words": (U64, [U64, U32]),
             "orc_log_encode": (None, [P, U64, U32, P]),
@@ -158,13 +163,17 @@ def rrr_set(off, nbr, model, seed, s):
     return out[:sz].copy()
 
 
-def sample(off, nbr, model, seed, first, count, nthreads=1, flags=0, per_set_edges=False):
+def sample(off, nbr, model, seed, first, count, nthreads=1, flags=0, per_set_edges=False, x=None):
     """Returns (offsets u64[count+1], members u32[total], edges_examined)
-    (edges_examined as u64[count], one per set, when per_set_edges)."""
+    (edges_examined as u64[count], one per set, when per_set_edges).
+    x: per-edge u32 probabilities p_e = (x_e + 1) / 2^32 (NEXT-3), None = WC."""
     off, nbr = _graph(off, nbr)
     n = off.size - 1
     L = _load()
-    if flags:
+    if x is not None:
+        xa = _weights(x, nbr)
+        a = L.orc_sample_w(n, _ptr(off), _ptr(nbr), _ptr(xa), MODELS[model], seed, first, count, flags, nthreads)
+    elif flags:
         a = L.orc_sample_ex(n, _ptr(off), _ptr(nbr), MODELS[model], seed, first, count, flags, nthreads)
     else:
         a = L.orc_sample(n, _ptr(off), _ptr(nbr), MODELS[model], seed, first, count, nthreads)
@@ -201,16 +210,41 @@ def imm_params(n, k, eps, ell):
     return p
 
 
-def imm(off, nbr, k, eps, ell, model, seed, nthreads=1, flags=0):
-    """Returns dict(seeds, theta, spread, stats).  flags: SOURCE_ELIM | FRESH_FINAL."""
+def _weights(x, nbr):
+    xa = np.ascontiguousarray(x, dtype=np.uint32)
+    return xa if xa.size else np.zeros(1, dtype=np.uint32)
+
+
+def ic_live_w(draw_, x):
+    return bool(_load().orc_ic_live_w(draw_, x))
+
+
+def lt_choice_w(tau, x_row):
+    """First j with sum_{i<=j}(x_i + 1) > tau, or None."""
+    xr = np.ascontiguousarray(x_row, dtype=np.uint32)
+    j = int(_load().orc_lt_choice_w(tau, _ptr(xr) if xr.size else None, xr.size))
+    return None if j == 0xFFFFFFFF else j
+
+
+def lt_weights_ok(off, x):
+    off = np.ascontiguousarray(off, dtype=np.uint64)
+    xa = np.ascontiguousarray(x, dtype=np.uint32)
+    return bool(_load().orc_lt_weights_ok(off.size - 1, _ptr(off), _ptr(xa) if xa.size else None))
+
+
+def imm(off, nbr, k, eps, ell, model, seed, nthreads=1, flags=0, x=None):
+    """Returns dict(seeds, theta, spread, stats).  flags: SOURCE_ELIM | FRESH_FINAL.
+    x: per-edge probabilities (NEXT-3), None = WC."""
     off, nbr = _graph(off, nbr)
     n = off.size - 1
     seeds = np.zeros(k, dtype=np.uint32)
     theta = ctypes.c_uint64()
     spread = ctypes.c_double()
     st = ImmStats()
-    rc = _load().orc_imm_ex(n, _ptr(off), _ptr(nbr), k, eps, ell, MODELS[model], seed, flags, nthreads,
-                            _ptr(seeds), ctypes.addressof(theta), ctypes.addressof(spread), ctypes.byref(st))
+    xa = _weights(x, nbr) if x is not None else None
+    rc = _load().orc_imm_w(n, _ptr(off), _ptr(nbr), _ptr(xa) if xa is not None else None, k, eps, ell,
+                           MODELS[model], seed, flags, nthreads,
+                           _ptr(seeds), ctypes.addressof(theta), ctypes.addressof(spread), ctypes.byref(st))
     if rc != 0:
         raise RuntimeError(f"orc_imm failed rc={rc}")
     rounds = min(st.rounds, 64)

@@ -25,6 +25,9 @@
  *                        path/star; enumeration of the retained-set law)
  *   fresh final phase .. pinned (estimation identical to the plain run;
  *                        final = greedy over ids from ORC_FRESH_BASE)
+ *   *_w (NEXT-3) ....... pinned (WC-derived weights reproduce the WC path;
+ *                        exact enumeration with general weights incl. the
+ *                        LT "no neighbour" outcome; boundary draws)
  *   orc_log_* .......... pinned (Fig. 1 example, hand-built containers,
  *                        numpy unpackbits layout, round trip)
  */
@@ -54,6 +57,13 @@ uint32_t orc_root(uint64_t seed, uint64_t s, uint32_t n);
 int      orc_ic_live(uint32_t draw, uint64_t d);      /* r <= p_vu with p = 1/d (R2) */
 uint32_t orc_lt_choice(uint32_t tau, uint64_t d);     /* prefix-scan choice (R3-R5) */
 
+/* general edge probabilities (NEXT-3, R25): p_e = (x_e + 1) / 2^32 */
+int      orc_ic_live_w(uint32_t draw, uint32_t x);
+/* first j with sum_{i<=j} (x_row[i] + 1) > tau, UINT32_MAX if none */
+uint32_t orc_lt_choice_w(uint32_t tau, const uint32_t* x_row, uint64_t d);
+/* every row's sum of (x_e + 1) <= 2^32 (LT: sum p <= 1) */
+int      orc_lt_weights_ok(uint32_t n, const uint64_t* off, const uint32_t* x);
+
 /* ---- one RRR set ------------------------------------------------------
  * Writes the members of RRR set `s` (ascending) to out[] (capacity n) and
  * returns the set size.  stamp[] is caller scratch of n uint64 that must be
@@ -78,6 +88,9 @@ orc_arena* orc_sample(uint32_t n, const uint64_t* off, const uint32_t* nbr, int 
  * possibly empty. */
 orc_arena* orc_sample_ex(uint32_t n, const uint64_t* off, const uint32_t* nbr, int model,
                          uint64_t seed, uint64_t first, uint64_t count, uint32_t flags, int nthreads);
+/* x: per-edge probabilities (R25), NULL = weighted cascade */
+orc_arena* orc_sample_w(uint32_t n, const uint64_t* off, const uint32_t* nbr, const uint32_t* x, int model,
+                        uint64_t seed, uint64_t first, uint64_t count, uint32_t flags, int nthreads);
 void       orc_arena_free(orc_arena* a);
 
 /* ---- greedy NodeSelection (Alg. 3) ------------------------- */
@@ -118,6 +131,10 @@ uint32_t orc_log_bits(uint64_t x_max);                 /* bit_width(x_max) */
 uint64_t orc_log_words(uint64_t count, uint32_t b);    /* 32-bit containers */
 void     orc_log_encode(const uint64_t* x, uint64_t count, uint32_t b, uint32_t* words);
 uint64_t orc_log_decode(const uint32_t* words, uint64_t j, uint32_t b);
+
+int orc_imm_w(uint32_t n, const uint64_t* off, const uint32_t* nbr, const uint32_t* x, uint32_t k, double eps,
+              double ell, int model, uint64_t seed, uint32_t flags, int nthreads,
+              uint32_t* seeds_out, uint64_t* theta_out, double* spread_out, orc_imm_stats* st);
 
 #ifdef __cplusplus
 }
