@@ -148,6 +148,23 @@ eim_status eim_graph_free(eim_graph* g);
 enum { EIM_G_LOG_ENCODE = 1u };
 eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
                                  const uint32_t* in_neighbors, uint32_t gflags, eim_graph** out);
+/* eim_load_graph_csr_weighted: general edge probabilities (NEXT-3; P:57
+ * "each edge (u,v) is assigned a random weight p_uv", P:61 LT "sum <= 1",
+ * P:377; R25).  edge_x[m] (host, borrowed; NULL = weighted
+ * cascade, i.e. eim_load_graph_csr_ex) gives in-edge e (the position in
+ * in_neighbors) the probability p_e = (edge_x[e] + 1) / 2^32; an edge with
+ * p = 0 must be left out of the graph.  IC: e is live iff its 32-bit draw
+ * <= edge_x[e].  LT: with w_j = edge_x[j] + 1 over a row, the first j with
+ * w_0 + ... + w_j > tau is chosen; none (the walk stops) if the row's sum
+ * <= tau.  LT needs every row's sum <= 2^32 (sum p <= 1): otherwise the
+ * graph loads but LT calls on it return EIM_E_INVAL.  The thresholds are
+ * streamed from HBM (4 B per examined in-edge, one 16-B load per Philox
+ * quad); LT keeps a per-edge cumulative array (+4 B per edge).
+ * Errors: those of eim_load_graph_csr_ex; EIM_E_INVAL for EIM_G_LOG_ENCODE
+ * together with edge_x. */
+eim_status eim_load_graph_csr_weighted(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                                       const uint32_t* in_neighbors, const uint32_t* edge_x, uint32_t gflags,
+                                       eim_graph** out);
 /* Device bytes held by the graph store (plain: 8(n+1) + 4 max(m,4) + 4n;
  * log-encoded: the two container arrays incl. 2 padding words each).
  * Errors: EIM_E_STATE (freed graph), EIM_E_INVAL (bytes NULL). */

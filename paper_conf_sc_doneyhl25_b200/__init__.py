@@ -30,7 +30,8 @@ STATUS_NAMES = {0: "EIM_OK", -1: "EIM_E_INVAL", -2: "EIM_E_NOMEM", -3: "EIM_E_CU
 
 # Every symbol include/eim.h declares (checked by tests/test_abi.py).
 EXPORTS = ["eim_create", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "eim_version",
-           "eim_load_graph_csr", "eim_load_graph_csr_ex", "eim_graph_bytes", "eim_graph_free", "eim_imm_run", "eim_imm_run_ex", "eim_sample_rrr",
+           "eim_load_graph_csr", "eim_load_graph_csr_ex", "eim_load_graph_csr_weighted", "eim_graph_bytes",
+           "eim_graph_free", "eim_imm_run", "eim_imm_run_ex", "eim_sample_rrr",
            "eim_sample_rrr_ex", "eim_select_seeds",
            "eim_imm_params", "eim_shard_range", "eim_get_stats"]
 
@@ -100,6 +101,7 @@ def lib():
         "eim_graph_free": (_I, [_P]),
         "eim_load_graph_csr_ex": (_I, [_P, _U32, _U64, _P, _P, _U32, ctypes.POINTER(_P)]),
         "eim_graph_bytes": (_I, [_P, ctypes.POINTER(_U64)]),
+        "eim_load_graph_csr_weighted": (_I, [_P, _U32, _U64, _P, _P, _P, _U32, ctypes.POINTER(_P)]),
         "eim_imm_run": (_I, [_P, _P, _U32, _D, _D, _I, _U64, _P, _P, _P, _P]),
         "eim_imm_run_ex": (_I, [_P, _P, _U32, _D, _D, _I, _U64, _U32, _P, _P, _P, _P]),
         "eim_sample_rrr": (_I, [_P, _P, _I, _U64, _U64, _U64, _P, _P, _U64, _P]),
@@ -155,15 +157,22 @@ def eim_last_error(ctx=None):
 
 
 # ------------------------------------------------------------------ graph
-def eim_load_graph_csr(ctx, in_offsets, in_neighbors, gflags=0):
+def eim_load_graph_csr(ctx, in_offsets, in_neighbors, gflags=0, edge_x=None):
     """in_offsets: u64[n+1] (numpy or pinned torch tensor .numpy()), in_neighbors: u32[m].
-    gflags != 0 (EIM_G_LOG_ENCODE) calls eim_load_graph_csr_ex."""
+    gflags != 0 (EIM_G_LOG_ENCODE) calls eim_load_graph_csr_ex; edge_x (u32[m], p = (x+1)/2^32)
+    calls eim_load_graph_csr_weighted."""
     off = _host(in_offsets, np.uint64)
     nbr = _host(in_neighbors, np.uint32)
     n = off.size - 1
     out = _P()
     args = (ctx, n, nbr.size, off.ctypes.data, nbr.ctypes.data if nbr.size else None)
-    if gflags:
+    if edge_x is not None:
+        x = _host(edge_x, np.uint32)
+        if x.size != nbr.size:
+            raise ValueError("edge_x must have one entry per edge")
+        _check(lib().eim_load_graph_csr_weighted(*args, x.ctypes.data if x.size else None, gflags,
+                                                 ctypes.byref(out)), ctx)
+    elif gflags:
         _check(lib().eim_load_graph_csr_ex(*args, gflags, ctypes.byref(out)), ctx)
     else:
         _check(lib().eim_load_graph_csr(*args, ctypes.byref(out)), ctx)

@@ -191,10 +191,17 @@ eim_status eim_load_graph_csr(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64
 
 eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
                                  const uint32_t* in_neighbors, uint32_t gflags, eim_graph** out) {
+  return eim_load_graph_csr_weighted(ctx, n, m, in_offsets, in_neighbors, nullptr, gflags, out);
+}
+
+eim_status eim_load_graph_csr_weighted(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
+                                       const uint32_t* in_neighbors, const uint32_t* edge_x, uint32_t gflags,
+                                       eim_graph** out) {
   if (!ctx_ok(ctx)) return EIM_E_STATE;
   return guarded(ctx, [&] {
     if (!out) fail(EIM_E_INVAL, "out is NULL");
     if (gflags & ~(uint32_t)EIM_G_LOG_ENCODE) fail(EIM_E_INVAL, "unknown graph flag");
+    if (edge_x && (gflags & EIM_G_LOG_ENCODE)) fail(EIM_E_INVAL, "EIM_G_LOG_ENCODE with edge probabilities is not supported");
     *out = nullptr;
     if (n < 2 || n >= 0xFFFFFFFFu) fail(EIM_E_INVAL, "n must be in [2, 2^32-1)");
     if (m >= (1ull << 40)) fail(EIM_E_INVAL, "m must be < 2^40");
@@ -219,11 +226,14 @@ eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uin
       g->bytes = ((uint64_t)n + 1) * sizeof(uint64_t) + std::max<uint64_t>(m, 4) * sizeof(uint32_t) +
                  (uint64_t)n * sizeof(uint32_t);
       if (gflags & EIM_G_LOG_ENCODE) graph_log_encode(ctx, g);
+      if (edge_x) graph_attach_weights(ctx, g, edge_x);
     } catch (...) {
       if (g->d_off) cudaFreeAsync(g->d_off, st);
       if (g->d_nbr) cudaFreeAsync(g->d_nbr, st);
       if (g->d_thr) cudaFreeAsync(g->d_thr, st);
       if (g->d_offw) cudaFreeAsync(g->d_offw, st);
+      if (g->d_x) cudaFreeAsync(g->d_x, st);
+      if (g->d_cum) cudaFreeAsync(g->d_cum, st);
       if (g->d_nbrw) cudaFreeAsync(g->d_nbrw, st);
       cudaStreamSynchronize(st);
       g->magic = 0;
@@ -241,11 +251,11 @@ eim_status eim_graph_free(eim_graph* g) {
     // every kernel that reads the graph has finished when a hot-path call
     // returns (the calls end synchronised), so the free is stream-ordered
     cudaSetDevice(ctx->device);
-    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw})
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum})
       if (p) cudaFreeAsync(p, ctx->stream);
     cudaStreamSynchronize(ctx->stream);
   } else {
-    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw})
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum})
       if (p) cudaFree(p);
   }
   g->magic = 0;
@@ -283,6 +293,7 @@ eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double e
     if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
     if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
+    if (model == EIM_LT && !g->lt_ok) fail(EIM_E_INVAL, "LT: a row's edge weights sum to more than 1");
     imm_run(ctx, g, k, eps, ell, model, seed, flags, seeds_out, theta_out, spread_out, &ctx->last_stats);
     if (stats_out) *stats_out = ctx->last_stats;
   });
@@ -305,6 +316,7 @@ eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, 
     if (flags & ~(uint32_t)EIM_F_SOURCE_ELIM) fail(EIM_E_INVAL, "unknown flag");
     if (!offsets_out || !members_total) fail(EIM_E_INVAL, "NULL output");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
+    if (model == EIM_LT && !g->lt_ok) fail(EIM_E_INVAL, "LT: a row's edge weights sum to more than 1");
     if (first_id + count < first_id || first_id + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids must be < 2^62");
     cudaStream_t st = ctx->stream;
     const auto t0 = std::chrono::steady_clock::now();

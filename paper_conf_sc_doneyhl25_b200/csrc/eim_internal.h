@@ -52,6 +52,20 @@ struct PackedGraphView {
   uint32_t boff, bnbr;
 };
 
+// Reverse CSR with general edge probabilities (NEXT-3, R25): in-edge e has
+// p_e = (x_e + 1) / 2^32.  IC: live iff draw <= x_e.  LT: cum_e = (sum of
+// w_i = x_i + 1 over the row up to and including e) - 1, so the choice is the
+// first e of the row with cum_e >= tau (none if tau > the row's last cum).
+// x is padded with zeros to a multiple of 4 entries (quad loads).
+struct WeightedGraphView {
+  uint32_t n;
+  uint64_t m;
+  const uint64_t* off;
+  const uint32_t* nbr;
+  const uint32_t* x;    // m (padded to 4): IC thresholds
+  const uint32_t* cum;  // m: LT inclusive cumulative weights - 1 (valid when the graph's lt_ok)
+};
+
 // Per-launch control block (device memory).  The counters that every group
 // polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
@@ -109,6 +123,11 @@ struct eim_graph {
   eim::PackedGraphView pview{};
   void* d_offw = nullptr;
   void* d_nbrw = nullptr;
+  bool weighted = false;         // general edge probabilities (eim_load_graph_csr_weighted): wview, d_x, d_cum
+  eim::WeightedGraphView wview{};
+  void* d_x = nullptr;
+  void* d_cum = nullptr;
+  bool lt_ok = true;             // weighted: every row's weights sum to <= 2^32 (LT usable)
   uint64_t bytes = 0;            // device bytes of the store
   int proper_edge = -1;  // has an edge u -> v, u != v (1/0; -1 = not yet computed)
 };
@@ -153,6 +172,8 @@ constexpr uint32_t SENTINEL = 0xFFFFFFFFu;
 void graph_validate_and_thresholds(eim_ctx* ctx, eim_graph* g);
 // Replace the plain store by its log encoding (frees off/nbr/thr).
 void graph_log_encode(eim_ctx* ctx, eim_graph* g);
+// Attach per-edge probabilities x (host, m entries) to a validated plain store.
+void graph_attach_weights(eim_ctx* ctx, eim_graph* g, const uint32_t* h_x);
 bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g);
 
 // ---- sample.cu

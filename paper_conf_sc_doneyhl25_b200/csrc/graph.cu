@@ -86,7 +86,59 @@ __global__ void max_of_kernel(const uint32_t* __restrict__ x, uint64_t count, un
   if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
 }
 
+// LT cumulative weights (R25): one warp per row, inclusive scan of
+// w = x + 1 in 64 bits; cum = scan - 1.  A row whose sum exceeds 2^32
+// (sum p > 1) raises *bad (LT is then rejected on this graph).
+__global__ void lt_cum_kernel(const uint64_t* __restrict__ off, const uint32_t* __restrict__ x, uint32_t n,
+                              uint32_t* __restrict__ cum, unsigned int* bad) {
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t v = warp; v < n; v += nwarps) {
+    const uint64_t e0 = off[v], e1 = off[v + 1];
+    unsigned long long carry = 0;
+    for (uint64_t b = e0; b < e1; b += 32) {
+      const uint64_t e = b + lane;
+      unsigned long long s = e < e1 ? (unsigned long long)x[e] + 1ull : 0ull;
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long t = __shfl_up_sync(0xFFFFFFFFu, s, o);
+        if (lane >= (uint32_t)o) s += t;
+      }
+      s += carry;
+      if (e < e1) {
+        if (s > (1ull << 32)) atomicOr(bad, 1u);
+        cum[e] = s > (1ull << 32) ? 0xFFFFFFFFu : (uint32_t)(s - 1ull);
+      }
+      carry = __shfl_sync(0xFFFFFFFFu, s, 31);
+    }
+  }
+}
+
 }  // namespace
+
+void graph_attach_weights(eim_ctx* ctx, eim_graph* g, const uint32_t* h_x) {
+  cudaStream_t st = ctx->stream;
+  const uint64_t m = g->view.m, m4 = (m + 3) / 4 * 4 + 4;
+  EIM_CUDA(cudaMallocAsync(&g->d_x, m4 * sizeof(uint32_t), st));
+  EIM_CUDA(cudaMallocAsync(&g->d_cum, std::max<uint64_t>(m, 1) * sizeof(uint32_t), st));
+  EIM_CUDA(cudaMemsetAsync(g->d_x, 0, m4 * sizeof(uint32_t), st));
+  if (m) EIM_CUDA(cudaMemcpyAsync(g->d_x, h_x, m * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+  ctx->scratch.reserve(1 << 20, false, st);
+  unsigned int* d_bad = reinterpret_cast<unsigned int*>(ctx->scratch.p);
+  EIM_CUDA(cudaMemsetAsync(d_bad, 0, sizeof(unsigned int), st));
+  lt_cum_kernel<<<grid_for(ctx, (uint64_t)g->view.n * 32, 256), 256, 0, st>>>(
+      g->view.off, static_cast<const uint32_t*>(g->d_x), g->view.n, static_cast<uint32_t*>(g->d_cum), d_bad);
+  EIM_CUDA(cudaGetLastError());
+  ctx->kernel_launches++;
+  unsigned int* h = static_cast<unsigned int*>(ctx->h_pinned);
+  EIM_CUDA(cudaMemcpyAsync(h, d_bad, sizeof(unsigned int), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+  g->lt_ok = *h == 0;
+  g->weighted = true;
+  g->wview = WeightedGraphView{g->view.n, m, g->view.off, g->view.nbr, static_cast<const uint32_t*>(g->d_x),
+                               static_cast<const uint32_t*>(g->d_cum)};
+  g->bytes += (m4 + std::max<uint64_t>(m, 1)) * sizeof(uint32_t);
+}
 
 uint32_t bit_width(uint64_t x) {
   uint32_t b = 0;
@@ -145,6 +197,7 @@ bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g) {
     EIM_CUDA(cudaMemsetAsync(d, 0, sizeof(unsigned int), st));
     const uint32_t grid = grid_for(ctx, (uint64_t)g->view.n * 32, 256);
     if (g->packed) proper_edge_kernel<<<grid, 256, 0, st>>>(g->pview, g->view.n, d);
+    else if (g->weighted) proper_edge_kernel<<<grid, 256, 0, st>>>(g->wview, g->view.n, d);
     else proper_edge_kernel<<<grid, 256, 0, st>>>(g->view, g->view.n, d);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches += 1;

@@ -39,4 +39,47 @@ __device__ __forceinline__ uint32_t g_thr(const PackedGraphView&, uint32_t, uint
   return (d == 0 || d > 0xFFFFFFFFull) ? 0u : 0xFFFFFFFFu / (uint32_t)d;
 }
 
+__device__ __forceinline__ uint64_t g_off(const WeightedGraphView& g, uint64_t v) { return g.off[v]; }
+__device__ __forceinline__ uint32_t g_nbr(const WeightedGraphView& g, uint64_t e) { return g.nbr[e]; }
+__device__ __forceinline__ uint32_t g_thr(const WeightedGraphView&, uint32_t, uint64_t) { return 0u; }
+
+// ---- IC liveness of the 4 edges of Philox quad q (words w): edge 4q+i is
+// live iff w_i <= its threshold.  Weighted cascade: one threshold T per row.
+template <class GV>
+__device__ __forceinline__ uint32_t quad_live_mask(const GV&, uint64_t, uint32_t T, const uint4& w) {
+  return (w.x <= T ? 1u : 0u) | (w.y <= T ? 2u : 0u) | (w.z <= T ? 4u : 0u) | (w.w <= T ? 8u : 0u);
+}
+template <class GV>
+__device__ __forceinline__ bool quad_any_live(const GV&, uint64_t, uint32_t T, const uint4& w) {
+  return min(min(w.x, w.y), min(w.z, w.w)) <= T;
+}
+// general probabilities: the quad's 4 thresholds in one 16-byte load
+__device__ __forceinline__ uint32_t quad_live_mask(const WeightedGraphView& g, uint64_t q, uint32_t, const uint4& w) {
+  const uint4 t = __ldg(reinterpret_cast<const uint4*>(g.x) + q);
+  return (w.x <= t.x ? 1u : 0u) | (w.y <= t.y ? 2u : 0u) | (w.z <= t.z ? 4u : 0u) | (w.w <= t.w ? 8u : 0u);
+}
+__device__ __forceinline__ bool quad_any_live(const WeightedGraphView& g, uint64_t q, uint32_t T, const uint4& w) {
+  return quad_live_mask(g, q, T, w) != 0u;
+}
+
+// ---- LT choice in row [e0, e1) for threshold tau: the offset j of the
+// chosen in-edge, or ~0 when no in-neighbour is chosen.  Weighted cascade
+// (R4): j = floor(tau d / 2^32).
+template <class GV>
+__device__ __forceinline__ uint64_t lt_choose(const GV&, uint64_t e0, uint64_t e1, uint32_t tau) {
+  return __umul64hi((unsigned long long)tau << 32, e1 - e0);
+}
+// general weights (R25): first e with cum_e >= tau (binary search; cum is
+// strictly increasing within the row)
+__device__ __forceinline__ uint64_t lt_choose(const WeightedGraphView& g, uint64_t e0, uint64_t e1, uint32_t tau) {
+  if (g.cum[e1 - 1] < tau) return ~0ull;
+  uint64_t lo = e0, hi = e1 - 1;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (g.cum[mid] >= tau) hi = mid;
+    else lo = mid + 1;
+  }
+  return lo - e0;
+}
+
 }  // namespace eim

@@ -330,10 +330,10 @@ template <int G, class GV>
 __device__ __forceinline__ void park_live(const GV& g, const RoundView& R, SampleCtl* ctl, const SG<G>& o,
                                        const Cur& c, uint4 w, uint32_t s_local, uint32_t head, uint32_t W) {
   const GroupRows<G>& rw = *o.rw;
-  uint32_t live = (w.x <= c.T ? 1u : 0u) | (w.y <= c.T ? 2u : 0u) | (w.z <= c.T ? 4u : 0u) | (w.w <= c.T ? 8u : 0u);
+  const unsigned long long q = ((unsigned long long)c.qhi << 32) | c.qlo;
+  uint32_t live = quad_live_mask(g, q, c.T, w);
   if (c.j == c.qe - rw.nq[c.r]) live &= 0xFu << rw.wlo[c.r];
   if (c.j == c.qe - 1u) live &= 0xFu >> (3u - rw.whi[c.r]);
-  const unsigned long long q = ((unsigned long long)c.qhi << 32) | c.qlo;
   while (live) {
     const int i = __ffs(live) - 1;
     live &= live - 1;
@@ -379,7 +379,8 @@ __device__ __forceinline__ void sweep_runs(const GV& g, const RoundView& R, Samp
     for (int k = 0; k < U; ++k) w[k] = edge_draws<HOIST>(c[k], E, c2, c3, R.K);
 #pragma unroll
     for (int k = 0; k < U; ++k)
-      if ((k == 0 || i < n[k]) && min4(w[k]) <= c[k].T) park_live<G>(g, R, ctl, o, c[k], w[k], s_local, head, W);
+      if ((k == 0 || i < n[k]) && quad_any_live(g, ((unsigned long long)c[k].qhi << 32) | c[k].qlo, c[k].T, w[k]))
+        park_live<G>(g, R, ctl, o, c[k], w[k], s_local, head, W);
     if (++i >= sub) break;
 #pragma unroll
     for (int k = 0; k < U; ++k)
@@ -823,7 +824,8 @@ __global__ void __launch_bounds__(256) lt_kernel(GV g, RoundView R, uint64_t cou
       ++steps;
       const uint4 w = philox_at((uint64_t)(u >> 2), s, TAG_LT, K);
       const uint32_t tau = word_of(w, u & 3u);
-      const unsigned long long j = __umul64hi((unsigned long long)tau << 32, e1 - e0);
+      const unsigned long long j = lt_choose(g, e0, e1, tau);
+      if (j == ~0ull) break;  // general weights: no in-neighbour activated (R25)
       const uint32_t v = g_nbr(g, e0 + j);
       const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
       if (ins == 0) break;
@@ -1053,6 +1055,8 @@ static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint
   const uint32_t W = ring_w();
   const size_t smem = ic_smem<G, NSG>(W);
   if (g->packed) launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, PackedGraphView>, g->pview, R, count, ctl, st, spare_sm_slot, W, smem);
+  else if (g->weighted)
+    launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, WeightedGraphView>, g->wview, R, count, ctl, st, spare_sm_slot, W, smem);
   else launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, GraphView>, g->view, R, count, ctl, st, spare_sm_slot, W, smem);
 }
 
@@ -1088,6 +1092,7 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
     uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
     const uint32_t grid = (uint32_t)std::max<uint64_t>(blocks, 1);
     if (g->packed) lt_kernel<<<grid, 256, 0, st>>>(g->pview, R, rd.count, ctl);
+    else if (g->weighted) lt_kernel<<<grid, 256, 0, st>>>(g->wview, R, rd.count, ctl);
     else lt_kernel<<<grid, 256, 0, st>>>(g->view, R, rd.count, ctl);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
@@ -1109,11 +1114,14 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
     // for half of that.  Consumers zero the descriptors they take, so
     // only fresh or abandoned memory needs a memset (the pool is written
     // before its descriptor is published).
+    const uint64_t old_pcap = rd.pcap;
     rd.pcap = 1ull << (rd.bits - 1);
     rd.tcap = rd.pcap / 2;
     void* before = rd.queue.p;
     rd.queue.reserve(4ull * rd.pcap + 16ull * rd.tcap, false, st);
-    if (rd.queue.p != before) rd.qdirty = true;
+    // the descriptors start at 4 * pcap: with another pool size they lie where
+    // an earlier round's pool (non-zero seed ids) may have been
+    if (rd.queue.p != before || rd.pcap != old_pcap) rd.qdirty = true;
     if (rd.qdirty) {
       EIM_CUDA(cudaMemsetAsync(static_cast<char*>(rd.queue.p) + 4ull * rd.pcap, 0, 16ull * rd.tcap, st));
       rd.qdirty = false;
@@ -1328,6 +1336,7 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
         rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_sum, roots, kidx);
   };
   if (g->packed) scatter(g->pview);
+  else if (g->weighted) scatter(g->wview);
   else scatter(g->view);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;

@@ -377,3 +377,110 @@ def test_log_encoded_C2_imm(eim, ctx, graphs):
         _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
     finally:
         eim.eim_graph_free(g)
+
+
+# NEXT-3: general edge probabilities (R25), thresholds streamed per edge.
+def _random_x(off, model, seed, frac_sum=0.9):
+    """Random per-edge x: IC p uniform in (0, 1]; LT a random split of mass <= 1 per row."""
+    rng = np.random.default_rng(seed)
+    m = int(off[-1])
+    if model == "IC":
+        return rng.integers(0, 2**32, size=m, dtype=np.uint64).astype(np.uint32)
+    d = np.diff(off).astype(np.int64)
+    row = np.repeat(np.arange(d.size), d)
+    r = rng.random(m) + 1e-3
+    rowsum = np.bincount(row, weights=r, minlength=d.size)
+    total = np.where(np.arange(d.size) % 3 != 0, np.floor(frac_sum * 2**32), 2.0**32)
+    w = np.floor(r / rowsum[row] * (total[row] - d[row])).astype(np.int64) + 1   # row sum <= total
+    x = (w - 1).astype(np.uint32)
+    return x
+
+
+def _weighted_equal(eim, ctx, off, nbr, x, model, seed, first, count, imm_args=None):
+    g = eim.eim_load_graph_csr(ctx, off, nbr, edge_x=x)
+    try:
+        go, gm = eim.eim_sample_rrr(ctx, g, model, seed, first, count)
+        ro, rm, rex = oracle.sample(off, nbr, model, seed, first, count, nthreads=NT, x=x)
+        assert np.array_equal(go, ro) and np.array_equal(gm, rm), (model, first, count)
+        assert eim.eim_get_stats(ctx)["edges_examined"] == rex
+        if imm_args:
+            k, eps, flags = imm_args
+            seeds, theta, spread, st = eim.eim_imm_run(ctx, g, k, eps, 1.0, model, seed, flags=flags)
+            ref = oracle.imm(off, nbr, k, eps, 1.0, model, seed, nthreads=NT, flags=flags, x=x)
+            assert np.array_equal(seeds, ref["seeds"]) and theta == ref["theta"] and spread == ref["spread"]
+            for key in ("theta_i", "cov_i", "edges_examined", "arena_elems", "ids_sampled"):
+                assert st[key] == ref[key], key
+    finally:
+        eim.eim_graph_free(g)
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_weighted_C1(eim, ctx, graphs, model, spill_mode):
+    off, nbr = graphs("C1")
+    for seed in (1, 2):
+        x = _random_x(off, model, seed)
+        if model == "IC":
+            x = (x >> np.uint32(4)).astype(np.uint32)  # p ~ U(0, 1/16): sets of moderate size
+        _weighted_equal(eim, ctx, off, nbr, x, model, seed, 0, 6000, (5, 0.5, 0))
+    _weighted_equal(eim, ctx, off, nbr, _random_x(off, model, 3) >> np.uint32(5), model, 3, 2**44 + 1, 333,
+                    (3, 0.3, ELIM))
+
+
+def test_weighted_special_cases(eim, ctx):
+    # p = 1 on a path: every set is a prefix; WC-derived weights on C1 reproduce the WC sets
+    off, nbr = inputs.path_graph(300)
+    x = np.full(nbr.size, 2**32 - 1, dtype=np.uint32)
+    for model in ("IC", "LT"):
+        _weighted_equal(eim, ctx, off, nbr, x, model, 4, 0, 500, (2, 0.5, 0))
+    off, nbr = inputs.config_graph("C1")
+    d = np.diff(off).astype(np.uint64)
+    row = np.repeat(np.arange(off.size - 1), d.astype(np.int64))
+    x_ic = (np.uint64(2**32 - 1) // d[row]).astype(np.uint32)
+    g = eim.eim_load_graph_csr(ctx, off, nbr, edge_x=x_ic)
+    try:
+        a = eim.eim_sample_rrr(ctx, g, "IC", 5, 0, 4000)
+        b = oracle.sample(off, nbr, "IC", 5, 0, 4000, nthreads=NT)
+        assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    finally:
+        eim.eim_graph_free(g)
+    # LT weights summing above 1 are rejected for LT, accepted for IC
+    off, nbr = inputs.from_edges(3, [(0, 2), (1, 2)])
+    g = eim.eim_load_graph_csr(ctx, off, nbr, edge_x=np.array([2**31, 2**31 - 1], dtype=np.uint32))
+    try:
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_imm_run(ctx, g, 1, 0.5, 1.0, "LT", 1)
+        assert ei.value.status == eim.EIM_E_INVAL
+        eim.eim_imm_run(ctx, g, 1, 0.5, 1.0, "IC", 1)
+    finally:
+        eim.eim_graph_free(g)
+    with pytest.raises(eim.EimError):
+        eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC, edge_x=np.zeros(2, dtype=np.uint32))
+
+
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_weighted_C2(eim, ctx, graphs, model):
+    off, nbr = graphs("C2")
+    x = _random_x(off, model, 7)
+    if model == "IC":  # trivalency-like small probabilities keep the sets moderate
+        x = (x >> np.uint32(6)).astype(np.uint32)
+    _weighted_equal(eim, ctx, off, nbr, x, model, 1, 0, 3000 if model == "IC" else 20000)
+
+
+def test_task_pool_layout_change_between_rounds(eim, ctx, graphs, monkeypatch):
+    # Regression: a round with a smaller task pool than the previous one (same
+    # buffer) must not read the previous pool's seed ids as task descriptors.
+    off, nbr = graphs("C2")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        with monkeypatch.context() as mp:
+            mp.setenv("EIM_TABLE_BITS", "26")
+            mp.setenv("EIM_SPILL_QUADS", "1")
+            mp.setenv("EIM_TASK_QUADS", "1")
+            _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 0, 3000)
+        with monkeypatch.context() as mp:
+            mp.setenv("EIM_SPILL_QUADS", "1")
+            mp.setenv("EIM_TASK_QUADS", "1")
+            _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 7000, 2000)
+        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 20000, 1000)
+    finally:
+        eim.eim_graph_free(g)
