@@ -289,10 +289,21 @@ def main():
     variants = []
     if args.variant_steps > 0 and world == 1:
         g_packed = eim.eim_load_graph_csr(ctx, off, nbr, gflags=eim.EIM_G_LOG_ENCODE)
-        for name, gv, flags in (("log_encoded_store", g_packed, 0),
-                                ("source_elim", g, eim.EIM_F_SOURCE_ELIM),
-                                ("source_elim+log_encoded_store", g_packed, eim.EIM_F_SOURCE_ELIM),
-                                ("fresh_final", g, eim.EIM_F_FRESH_FINAL)):
+        # NEXT-3 layout: the weighted-cascade probabilities given as per-edge
+        # thresholds (R25), streamed from HBM -- same results as the plain run
+        d = np.diff(off).astype(np.uint64)
+        if c["model"] == "IC":
+            x_wc = (np.uint64(2**32 - 1) // np.repeat(d, d.astype(np.int64))).astype(np.uint32)
+        else:
+            x_wc = None  # LT: the WC run needs no weights; the general LT path is covered by the parity tests
+        g_w = eim.eim_load_graph_csr(ctx, off, nbr, edge_x=x_wc) if x_wc is not None else None
+        runs = [("log_encoded_store", g_packed, 0),
+                ("source_elim", g, eim.EIM_F_SOURCE_ELIM),
+                ("source_elim+log_encoded_store", g_packed, eim.EIM_F_SOURCE_ELIM),
+                ("fresh_final", g, eim.EIM_F_FRESH_FINAL)]
+        if g_w is not None:
+            runs.append(("per_edge_thresholds", g_w, 0))
+        for name, gv, flags in runs:
             for _ in range(2):
                 eim.eim_imm_run(ctx, gv, c["k"], c["eps"], c["ell"], c["model"], RUN_SEED, flags=flags)
             vms, vst = 0.0, None
@@ -308,12 +319,22 @@ def main():
             vms /= args.variant_steps
             variants.append({"variant": name, "ms_per_step": vms, "rrr_sets_per_s": vth / (vms / 1e3),
                              "theta": vth, "ids_sampled": vst["ids_sampled"], "arena_elems": vst["arena_elems"],
-                             "arena_bytes": 4 * vst["arena_elems"], "graph_bytes": eim.eim_graph_bytes(gv),
+                             "arena_bytes": vst["arena_bytes"], "graph_bytes": eim.eim_graph_bytes(gv),
                              "edges_examined": vst["edges_examined"],
                              "sample_kernel_ms": vst["ms_sample_kernel"], "select_ms": vst["ms_select"],
                              "seeds_head": vs[:5].tolist(),
                              "seeds_equal_plain": bool(np.array_equal(vs, seeds)) if flags == 0 else None})
+            if name == "per_edge_thresholds" and vst["ms_sample_kernel"] > 0:
+                # 4 B of threshold per examined in-edge streamed from HBM (plus the
+                # WC path's per-vertex bytes): the HBM-bound layout of SURVEY §8(d)
+                gbs = 4.0 * vst["edges_examined"] / (vst["ms_sample_kernel"] / 1e3) / 1e9
+                hbm = float(_peaks().get("hbm_gbs", 8000.0))
+                variants[-1]["threshold_stream_gbs"] = gbs
+                variants[-1]["threshold_stream_frac_hbm"] = gbs / hbm
+                variants[-1]["edges_per_s"] = vst["edges_examined"] / (vst["ms_sample_kernel"] / 1e3)
         eim.eim_graph_free(g_packed)
+        if g_w is not None:
+            eim.eim_graph_free(g_w)
     budget = None
     if args.budget_ids > 0:
         lo_b, hi_b = eim.eim_shard_range(0, args.budget_ids, rank, world)
@@ -372,7 +393,7 @@ def main():
                     "h2d_bytes_per_step": int(off.nbytes + nbr.nbytes), "d2h_bytes_per_step": int(4 * c["k"] + 16),
                     "ms_per_step": e2e_ms_step},
             "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
-            "memory": {"graph_bytes": eim.eim_graph_bytes(g), "arena_bytes": 4 * stats[-1]["arena_elems"],
+            "memory": {"graph_bytes": eim.eim_graph_bytes(g), "arena_bytes": stats[-1]["arena_bytes"],
                        "graph_bytes_log_encoded": next((v["graph_bytes"] for v in variants
                                                         if v["variant"] == "log_encoded_store"), None)},
             "variants": variants,
