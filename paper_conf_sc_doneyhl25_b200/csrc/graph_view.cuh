@@ -7,8 +7,10 @@
 
 namespace eim {
 
-__device__ __forceinline__ uint64_t g_off(const GraphView& g, uint64_t v) { return g.off[v]; }
-__device__ __forceinline__ uint32_t g_nbr(const GraphView& g, uint64_t e) { return g.nbr[e]; }
+// read-only path (ld.global.nc): the store never changes while a kernel runs,
+// and the loads may be issued ahead of the membership-table atomics
+__device__ __forceinline__ uint64_t g_off(const GraphView& g, uint64_t v) { return __ldg(g.off + v); }
+__device__ __forceinline__ uint32_t g_nbr(const GraphView& g, uint64_t e) { return __ldg(g.nbr + e); }
 __device__ __forceinline__ uint32_t g_thr(const GraphView& g, uint32_t v, uint64_t /*d*/) { return g.thr[v]; }
 
 // Value j of a log-encoded array (R24): bits [j b, (j+1) b) of the
@@ -39,8 +41,8 @@ __device__ __forceinline__ uint32_t g_thr(const PackedGraphView&, uint32_t, uint
   return (d == 0 || d > 0xFFFFFFFFull) ? 0u : 0xFFFFFFFFu / (uint32_t)d;
 }
 
-__device__ __forceinline__ uint64_t g_off(const WeightedGraphView& g, uint64_t v) { return g.off[v]; }
-__device__ __forceinline__ uint32_t g_nbr(const WeightedGraphView& g, uint64_t e) { return g.nbr[e]; }
+__device__ __forceinline__ uint64_t g_off(const WeightedGraphView& g, uint64_t v) { return __ldg(g.off + v); }
+__device__ __forceinline__ uint32_t g_nbr(const WeightedGraphView& g, uint64_t e) { return __ldg(g.nbr + e); }
 __device__ __forceinline__ uint32_t g_thr(const WeightedGraphView&, uint32_t, uint64_t) { return 0u; }
 
 // ---- IC liveness of the 4 edges of Philox quad q (words w): edge 4q+i is

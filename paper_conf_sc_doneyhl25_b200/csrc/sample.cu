@@ -815,23 +815,31 @@ __global__ void __launch_bounds__(256) lt_kernel(GV g, RoundView R, uint64_t cou
     const uint32_t s_local = (uint32_t)t;
     const uint64_t s = R.base + s_local;
     uint32_t u = draw_root(s, g.n, K);
+    // A step's critical path is off[u] -> nbr[e0 + j] -> the membership
+    // insert of v.  The insert only decides whether the walk stops, so v's
+    // row and threshold are loaded and drawn before its result is awaited:
+    // two dependent memory round trips per step instead of three.
+    unsigned long long e0 = g_off(g, u), e1 = g_off(g, u + 1);
+    uint32_t tau = word_of(philox_at((uint64_t)(u >> 2), s, TAG_LT, K), u & 3u);
     bool ok = table_insert(R.keys, R.bits, table_key(s_local, u)) >= 0;
     uint32_t L = 1;
     unsigned long long steps = 0;
     while (ok) {
-      const unsigned long long e0 = g_off(g, u), e1 = g_off(g, u + 1);
       if (e1 == e0) break;
       ++steps;
-      const uint4 w = philox_at((uint64_t)(u >> 2), s, TAG_LT, K);
-      const uint32_t tau = word_of(w, u & 3u);
       const unsigned long long j = lt_choose(g, e0, e1, tau);
       if (j == ~0ull) break;  // general weights: no in-neighbour activated (R25)
       const uint32_t v = g_nbr(g, e0 + j);
+      const unsigned long long f0 = g_off(g, v), f1 = g_off(g, v + 1);
+      const uint32_t tv = word_of(philox_at((uint64_t)(v >> 2), s, TAG_LT, K), v & 3u);
       const int ins = table_insert(R.keys, R.bits, table_key(s_local, v));
       if (ins == 0) break;
       if (ins < 0) ok = false;
       ++L;
       u = v;
+      e0 = f0;
+      e1 = f1;
+      tau = tv;
     }
     if (ok) {
       R.sizes[s_local] = L;
