@@ -3,7 +3,8 @@
 The library's N>1 path (imm.cpp sample_round) is: every round's new sample
 ids [|R|, theta_i) are split with eim_shard_range (the library's own host
 function, called here), each rank samples its share, the shares are
-exchanged in rank order (= sample-id order) and the greedy runs replicated.
+exchanged in rank order (= sample-id order) and the greedy runs replicated
+(also with the fresh final phase, whose ids start at EIM_FRESH_BASE).
 Here each rank samples with the oracle and exchanges over gloo; the result
 must equal the single-process oracle IMM bit for bit on every rank.
 """
@@ -29,8 +30,10 @@ def _free_port():
     return p
 
 
-def _dist_imm(rank, world, off, nbr, k, eps, ell, model, seed):
-    """Mirror of imm.cpp's control flow with the exchange done over gloo."""
+def _dist_imm(rank, world, off, nbr, k, eps, ell, model, seed, fresh=False):
+    """Mirror of imm.cpp's control flow with the exchange done over gloo.
+    fresh: the final phase draws theta sets from ids FRESH_BASE.. (R23),
+    sharded the same way (set index i = sample id FRESH_BASE + i)."""
     n = off.size - 1
     p = eim.eim_imm_params(n, k, eps, ell)
     offsets = [np.zeros(1, dtype=np.uint64)]
@@ -38,11 +41,12 @@ def _dist_imm(rank, world, off, nbr, k, eps, ell, model, seed):
     R, cov, total = 0, 0, 0
     LB = 1.0
     rounds = []
+    id_base = 0
 
     def sample_round(R, R_new):
         nonlocal total
         lo, hi = eim.eim_shard_range(R, R_new - R, rank, world)
-        o, m, _ = oracle.sample(off, nbr, model, seed, lo, hi - lo)
+        o, m, _ = oracle.sample(off, nbr, model, seed, id_base + lo, hi - lo)
         gathered = [None] * world
         dist.all_gather_object(gathered, (lo, hi, o, m))
         for q in range(world):  # rank order == sample-id order
@@ -74,6 +78,10 @@ def _dist_imm(rank, world, off, nbr, k, eps, ell, model, seed):
             break
         i += 1
     theta = int(np.ceil(p.lambda_s / LB))
+    if fresh:
+        offsets[:] = [np.zeros(1, dtype=np.uint64)]
+        members.clear()
+        total, R, R_sel, id_base = 0, 0, None, eim.EIM_FRESH_BASE
     if theta > R:
         sample_round(R, theta)
         R = theta
@@ -90,8 +98,9 @@ def _worker(rank, world, port, q):
         off, nbr = inputs.config_graph("C1")
         for model in ("IC", "LT"):
             for seed in (1, 2):
-                S, theta, spread, rounds = _dist_imm(rank, world, off, nbr, 5, 0.5, 1.0, model, seed)
-                out.append((model, seed, S.tolist(), theta, spread, rounds))
+                for fresh in (False, True):
+                    S, theta, spread, rounds = _dist_imm(rank, world, off, nbr, 5, 0.5, 1.0, model, seed, fresh)
+                    out.append((model, seed, fresh, S.tolist(), theta, spread, rounds))
         q.put((rank, out))
     finally:
         dist.destroy_process_group()
@@ -112,8 +121,8 @@ def test_multi_rank_protocol_matches_single_process(world):
         assert p_.exitcode == 0
     off, nbr = inputs.config_graph("C1")
     for r in range(world):
-        for (model, seed, S, theta, spread, rounds) in results[r]:
-            ref = oracle.imm(off, nbr, 5, 0.5, 1.0, model, seed)
+        for (model, seed, fresh, S, theta, spread, rounds) in results[r]:
+            ref = oracle.imm(off, nbr, 5, 0.5, 1.0, model, seed, flags=oracle.FRESH_FINAL if fresh else 0)
             assert S == ref["seeds"].tolist(), (r, model, seed)
             assert theta == ref["theta"] and spread == ref["spread"]
             assert [x for x, _ in rounds] == ref["theta_i"] and [c for _, c in rounds] == ref["cov_i"]
