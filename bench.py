@@ -332,6 +332,14 @@ def main():
                 variants[-1]["threshold_stream_gbs"] = gbs
                 variants[-1]["threshold_stream_frac_hbm"] = gbs / hbm
                 variants[-1]["edges_per_s"] = vst["edges_examined"] / (vst["ms_sample_kernel"] / 1e3)
+                if args.budget_ids > 0:  # the same layout on the fixed sample budget (no round tails)
+                    eim.eim_sample_rrr(ctx, gv, c["model"], RUN_SEED, 0, args.budget_ids)
+                    sb = eim.eim_get_stats(ctx)
+                    bgbs = 4.0 * sb["edges_examined"] / (sb["ms_sample_kernel"] / 1e3) / 1e9
+                    variants[-1]["fixed_budget"] = {
+                        "ids": args.budget_ids, "kernel_ms": sb["ms_sample_kernel"],
+                        "edges_per_s": sb["edges_examined"] / (sb["ms_sample_kernel"] / 1e3),
+                        "threshold_stream_gbs": bgbs, "threshold_stream_frac_hbm": bgbs / hbm}
         eim.eim_graph_free(g_packed)
         if g_w is not None:
             eim.eim_graph_free(g_w)
@@ -386,8 +394,11 @@ def main():
                           "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
                           "traffic": traffic,
                           "peak_basis": "28 algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
+            # IC: examined edges/s vs the Philox roof; LT: 28 algorithmic bytes per walk step vs HBM
             "sampler_fixed_budget": (dict(budget, frac=(budget["edges_per_s"] / 1e9 / world / peak)
-                                          if c["model"] == "IC" else None) if budget else None),
+                                          if c["model"] == "IC" else
+                                          (28.0 * budget["edges_per_s"] / 1e9 / world / peak))
+                                     if budget else None),
             "cpu_baseline": cb,
             "e2e": {"value": theta_all / (e2e_ms_step / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": int(off.nbytes + nbr.nbytes), "d2h_bytes_per_step": int(4 * c["k"] + 16),
