@@ -17,7 +17,7 @@ off, nbr = inputs.config_graph(cfg)
 ctx = eim.eim_create(0)
 g = eim.eim_load_graph_csr(ctx, off, nbr)
 ref = None
-for rq in ("0", "4096", "2048", "1024", "512", "256", "0", "2048"):
+for rq in ("0", "8192", "4096", "2048", "1024", "512", "0", "2048"):
     os.environ["EIM_ROW_TASK_QUADS"] = rq
     eim.eim_imm_run(ctx, g, c["k"], c["eps"], c["ell"], c["model"], 1)
     tot, ker = [], []
