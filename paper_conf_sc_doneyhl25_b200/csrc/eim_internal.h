@@ -70,7 +70,7 @@ struct WeightedGraphView {
 // polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
   unsigned long long ticket, pad0[15];          // next sample id (s_local)
-  unsigned long long thead, ttail, pad1[14];    // task descriptors: next to take, reserved
+  unsigned long long thead, ttail, pad1[14];    // tasks claimed / pushed over all queues (a hint for idle groups)
   unsigned long long ptail, pad2[15];           // task seed pool: reserved
   unsigned long long outstanding, pad3[15];     // samples + tasks taken or queued, not finished
   unsigned long long edges;                     // examined in-edges / walk steps (finalize)

@@ -165,7 +165,16 @@ struct RoundView {
   unsigned long long* dbg;       // [count][8] per root traversal (EIM_DEBUG_TIMELINE), nullable
   PhiloxKey K;                   // round keys of the seed (kernel parameter: read as constant operands)
   uint32_t nohoist;              // 1: never use the hoisted edge draws (tests exercise the general path)
+  unsigned long long* qc;        // task queue q: head at qc[16 q], tail at qc[16 q + 1] (one 128-B line each)
 };
+
+// Split-off tasks go to TQ queues (descriptor segments of tcap / TQ each):
+// a producer pushes to the queue of its block, a consumer claims from its
+// own queue first and then from the others.  With one queue every claim of
+// the round went through one CAS on one counter, about one claim per L2
+// round trip for the whole GPU, which bounded the heavy configs.
+constexpr uint32_t TQ = 16;
+__device__ __forceinline__ uint32_t home_queue() { return blockIdx.x % TQ; }
 
 constexpr uint32_t LIVE_CAP = 512;  // live in-edges parked per batch (more are visited inline)
 
@@ -230,8 +239,12 @@ __device__ __forceinline__ void task_write(const RoundView& R, unsigned long lon
 __device__ __forceinline__ void task_push1(const RoundView& R, SampleCtl* ctl, uint32_t s_local, uint32_t v) {
   atomicAdd(&ctl->outstanding, 1ull);
   const unsigned long long po = atomicAdd(&ctl->ptail, 1ull);
-  const unsigned long long ti = atomicAdd(&ctl->ttail, 1ull);
-  if (ti >= R.tcap) {  // descriptor array full: host redoes the round larger
+  const uint32_t q = home_queue();
+  const unsigned long long tq = R.tcap / TQ;
+  const unsigned long long qi = atomicAdd(&R.qc[16 * q + 1], 1ull);
+  atomicAdd(&ctl->ttail, 1ull);  // hint: tasks pushed (all queues)
+  const unsigned long long ti = q * tq + qi;
+  if (qi >= tq) {  // descriptor segment full: host redoes the round larger
     mark_fail(ctl);
     atomicAdd(&ctl->outstanding, ~0ull);
     return;
@@ -573,25 +586,26 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
       if (gtid == 0) {
         atomicAdd(&ctl->outstanding, (unsigned long long)ntasks);
         gc.base = atomicAdd(&ctl->ptail, (unsigned long long)npush);
-        gc.h = atomicAdd(&ctl->ttail, (unsigned long long)ntasks);
+        gc.h = atomicAdd(&R.qc[16 * home_queue() + 1], (unsigned long long)ntasks);  // index in the block's queue
+        atomicAdd(&ctl->ttail, (unsigned long long)ntasks);
         atomicAdd(&ctl->tasks_pushed, (unsigned long long)ntasks);
       }
       gsync<G>(gi);
-      const unsigned long long po = gc.base, ti = gc.h;
+      const unsigned long long po = gc.base, qi = gc.h, tq = R.tcap / TQ, ti = home_queue() * tq + qi;
       const bool ok = po + npush <= R.pcap;
       if (ok)
         for (uint32_t i = gtid; i < npush; i += G) R.pool[po + i] = me.ring[(head + tv + i) & (W - 1)];
       __threadfence();
       gsync<G>(gi);
       for (uint32_t t = gtid; t < ntasks; t += G) {
-        if (ti + t >= R.tcap) continue;
+        if (qi + t >= tq) continue;
         const uint32_t nv = min(tv, npush - t * tv);
         task_write(R, ti + t, po + (unsigned long long)t * tv, s_local, ok ? nv : 0u);
       }
       if (gtid == 0) {
-        if (!ok || ti + ntasks > R.tcap) {
+        if (!ok || qi + ntasks > tq) {
           mark_fail(ctl);
-          const unsigned long long lost = ti + ntasks > R.tcap ? ti + ntasks - max(ti, (unsigned long long)R.tcap) : 0;
+          const unsigned long long lost = qi + ntasks > tq ? qi + ntasks - max(qi, tq) : 0;
           if (lost) atomicAdd(&ctl->outstanding, 0ull - lost);
         }
         gc.tail = head + tv;
@@ -689,13 +703,26 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
 __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
   const volatile unsigned int* cp = R.cancel;
   if (cp[0] || cp[1]) return ACT_EXIT;  // cancelled or paused
-  unsigned long long h = vload(&ctl->thead);
-  for (;;) {
-    const unsigned long long t = min(vload(&ctl->ttail), (unsigned long long)R.tcap);
-    if (h >= t) break;
-    const unsigned long long old = atomicCAS(&ctl->thead, h, h + 1);
-    if (old == h) {
-      unsigned long long* d = R.tasks + 2 * h;
+  const unsigned long long tq = R.tcap / TQ;
+  const uint32_t home = home_queue();
+  // hint (pushed vs claimed, all queues): scan the queues only when some
+  // task may be waiting; a task missed here is seen by the next call (a
+  // group exits only when nothing is outstanding)
+  const bool any_task = vload(&ctl->ttail) > vload(&ctl->thead);
+  for (uint32_t k = 0; any_task && k < TQ; ++k) {
+    const uint32_t q = (home + k) % TQ;
+    unsigned long long* head = &R.qc[16 * q];
+    unsigned long long h = vload(head);
+    for (;;) {
+      const unsigned long long t = min(vload(head + 1), tq);
+      if (h >= t) break;
+      const unsigned long long old = atomicCAS(head, h, h + 1);
+      if (old != h) {
+        h = old;
+        continue;
+      }
+      atomicAdd(&ctl->thead, 1ull);
+      unsigned long long* d = R.tasks + 2 * (q * tq + h);
       unsigned long long w1;
       while ((w1 = vload(d + 1)) == 0ull) __nanosleep(32);  // claimed before it was written
       __threadfence();
@@ -706,7 +733,6 @@ __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, u
       gc.nb = (uint32_t)w1;
       return ACT_TASK;
     }
-    h = old;
   }
   if (vload(&ctl->ticket) < count) {
     atomicAdd(&ctl->outstanding, 1ull);  // before the ticket: an observer never sees "all taken, none outstanding" early
@@ -1069,6 +1095,13 @@ static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint
 }
 
 
+// the TQ task-queue counters follow the SampleCtl and the cancel/pause flags
+constexpr size_t QC_OFFSET = (sizeof(SampleCtl) + 16 + 127) / 128 * 128;
+constexpr size_t CTL_BYTES = QC_OFFSET + TQ * 128;
+static unsigned long long* round_queues(Round& rd) {
+  return reinterpret_cast<unsigned long long*>(static_cast<char*>(rd.ctl.p) + QC_OFFSET);
+}
+
 static RoundView round_view(Round& rd) {
   return RoundView{rd.table.as<unsigned long long>(),
                    rd.bits,
@@ -1082,7 +1115,8 @@ static RoundView round_view(Round& rd) {
                    rd.tcap,
                    rd.dbg.as<unsigned long long>(),
                    philox_key(rd.seed),
-                   std::getenv("EIM_NO_HOIST") ? 1u : 0u};
+                   std::getenv("EIM_NO_HOIST") ? 1u : 0u,
+                   round_queues(rd)};
 }
 
 // one sampler launch over rd's remaining work, bracketed by events
@@ -1124,7 +1158,7 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
     // before its descriptor is published).
     const uint64_t old_pcap = rd.pcap;
     rd.pcap = 1ull << (rd.bits - 1);
-    rd.tcap = rd.pcap / 2;
+    rd.tcap = rd.pcap / 2;  // TQ segments of tcap / TQ descriptors
     void* before = rd.queue.p;
     rd.queue.reserve(4ull * rd.pcap + 16ull * rd.tcap, false, st);
     // the descriptors start at 4 * pcap: with another pool size they lie where
@@ -1139,7 +1173,7 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
   }
   EIM_CUDA(cudaMemsetAsync(rd.sizes.p, 0, count * sizeof(uint32_t), st));
   EIM_CUDA(cudaMemsetAsync(rd.edges.p, 0, count * sizeof(unsigned long long), st));
-  EIM_CUDA(cudaMemsetAsync(rd.ctl.p, 0, sizeof(SampleCtl) + 16, st));
+  EIM_CUDA(cudaMemsetAsync(rd.ctl.p, 0, CTL_BYTES, st));
   if (std::getenv("EIM_DEBUG_TIMELINE")) {
     rd.dbg.reserve(64 * count, false, st);
     EIM_CUDA(cudaMemsetAsync(rd.dbg.p, 0, 64 * count, st));
@@ -1181,7 +1215,7 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   rd.edges.reserve(count * sizeof(unsigned long long), false, st);
   rd.fill.reserve(count * sizeof(uint32_t), false, st);
   rd.excl.reserve((count + 1) * sizeof(uint64_t), false, st);
-  rd.ctl.reserve(sizeof(SampleCtl) + 16, false, st);
+  rd.ctl.reserve(CTL_BYTES, false, st);
   // table capacity: >= 4x the expected members (mean set size of earlier
   // rounds, else 64), at least 2^20 slots
   const double mean = ctx->est_mean_size > 0 ? ctx->est_mean_size : 64.0;
