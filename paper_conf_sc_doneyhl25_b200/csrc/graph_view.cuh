@@ -45,6 +45,14 @@ __device__ __forceinline__ uint64_t g_off(const WeightedGraphView& g, uint64_t v
 __device__ __forceinline__ uint32_t g_nbr(const WeightedGraphView& g, uint64_t e) { return __ldg(g.nbr + e); }
 __device__ __forceinline__ uint32_t g_thr(const WeightedGraphView&, uint32_t, uint64_t) { return 0u; }
 
+// L2 prefetch of in_nbr[e] (no register result, so the sweep does not wait)
+__device__ __forceinline__ void l2_prefetch(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
+__device__ __forceinline__ void g_prefetch_nbr(const GraphView& g, uint64_t e) { l2_prefetch(g.nbr + e); }
+__device__ __forceinline__ void g_prefetch_nbr(const WeightedGraphView& g, uint64_t e) { l2_prefetch(g.nbr + e); }
+__device__ __forceinline__ void g_prefetch_nbr(const PackedGraphView& g, uint64_t e) {
+  l2_prefetch(g.nbrw + ((e * g.bnbr) >> 5));
+}
+
 // ---- IC liveness of the 4 edges of Philox quad q (words w): edge 4q+i is
 // live iff w_i <= its threshold.  Weighted cascade: one threshold T per row.
 template <class GV>

@@ -166,6 +166,7 @@ struct RoundView {
   PhiloxKey K;                   // round keys of the seed (kernel parameter: read as constant operands)
   uint32_t nohoist;              // 1: never use the hoisted edge draws (tests exercise the general path)
   unsigned long long* qc;        // task queue q: head at qc[16 q], tail at qc[16 q + 1] (one 128-B line each)
+  uint32_t prefetch;             // L2-prefetch in_nbr of parked live edges (EIM_NO_PREFETCH=1 turns it off)
 };
 
 // Split-off tasks go to TQ queues (descriptor segments of tcap / TQ each):
@@ -352,7 +353,10 @@ __device__ __forceinline__ void park_live(const GV& g, const RoundView& R, Sampl
     live &= live - 1;
     const unsigned long long e = (q << 2) + i;
     const uint32_t p = atomicAdd(&o.gc->nlive, 1u);
-    if (p < LIVE_CAP) o.live_e[p] = e;
+    if (p < LIVE_CAP) {
+      o.live_e[p] = e;
+      if (R.prefetch) g_prefetch_nbr(g, e);  // the visit phase reads nbr[e]: start it on its way to L2 now
+    }
     else visit_for<G>(g, R, ctl, o, s_local, head, W, g_nbr(g, e));
   }
 }
@@ -1116,7 +1120,8 @@ static RoundView round_view(Round& rd) {
                    rd.dbg.as<unsigned long long>(),
                    philox_key(rd.seed),
                    std::getenv("EIM_NO_HOIST") ? 1u : 0u,
-                   round_queues(rd)};
+                   round_queues(rd),
+                   std::getenv("EIM_NO_PREFETCH") ? 0u : 1u};
 }
 
 // one sampler launch over rd's remaining work, bracketed by events
