@@ -106,6 +106,7 @@ struct Round {
   cudaEvent_t ev[2 * MAX_LAUNCH] = {};  // start/stop of every sampler launch of the round
   int nlaunch = 0;
   bool launched = false;
+  bool waited = false;  // the launch has finished (round_finalize with keep appends the rest later)
   bool hist = true;
   uint32_t rflags = 0;
 };
@@ -198,7 +199,10 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 // Wait for rd, redo what overflowed, and append its first `use` sets to the
 // arena (sample-id order) with their histogram.  With RF_DROP_EMPTY, `use`
 // is the number of non-empty sets wanted (res.kept <= use, res.consumed ids).
-SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use);
+// from/keep: append only s_local in [from, use) and keep the round for a
+// later append of the rest (plain rounds; the IMM driver's lookahead).
+SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from = 0,
+                            bool keep = false);
 // Stop a launched speculative round and wait for it.
 void round_cancel(eim_ctx* ctx, Round& rd);
 // Let a launched round take no new sample ids (its running samples finish);

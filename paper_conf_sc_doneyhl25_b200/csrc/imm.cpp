@@ -121,11 +121,19 @@ class RoundSampler {
     // opt-in (EIM_SPECULATE=1): measured on C2 the speculative round slows the
     // current round's critical chains as much as it fills their idle SMs
     speculate_ = ctx->world == 1 && !elim && std::getenv("EIM_SPECULATE") != nullptr;
+    // Lookahead (default on, one GPU, plain runs): when the next round adds no
+    // more ids than this one, one launch samples both and the next round's
+    // sets are appended from the same round table without a launch -- one
+    // round tail (the heavy samples' critical paths) instead of two.  Sample
+    // ids are fixed labels, so the sets are the same; if the estimation loop
+    // stops first, the extra sets are discarded.  EIM_NO_LOOKAHEAD=1: off.
+    lookahead_ = ctx->world == 1 && !elim && !speculate_ && std::getenv("EIM_NO_LOOKAHEAD") == nullptr;
   }
 
   // Continue with an empty arena from sample id `id_base` (fresh final phase, R23).
   void restart(uint64_t id_base) {
     cancel();
+    drop_held();
     id_base_ = next_id_ = id_base;
   }
   ~RoundSampler() {
@@ -147,6 +155,11 @@ class RoundSampler {
     if (ctx_->world > 1) {
       sample_round(ctx_, g_, model_, seed_, id_base_, R, to, st_, ex_);
       R = to;
+      return;
+    }
+    if (lookahead_) {
+      grow_lookahead(R, to, next_to);
+      st_->ms_sample += ms_since(t0);
       return;
     }
     Round* cur = nullptr;
@@ -185,6 +198,7 @@ class RoundSampler {
       round_cancel(ctx_, *spec_);
       spec_ = nullptr;
     }
+    drop_held();
   }
 
  private:
@@ -195,6 +209,45 @@ class RoundSampler {
     st_->sample_launches += r.launches;
     st_->ms_sample_kernel += r.kernel_ms;
   }
+  // The held launch covers ids id_base_ + [held_first_, held_end_); sets
+  // [held_first_, held_done_) are appended.
+  void grow_lookahead(uint64_t& R, uint64_t to, uint64_t next_to) {
+    Round& rd = ctx_->rounds[0];
+    if (held_) {
+      if (held_done_ == R) {
+        const uint64_t upto = std::min(held_end_, to);
+        const bool keep = upto < held_end_;
+        account(round_finalize(ctx_, g_, rd, upto - held_first_, held_done_ - held_first_, keep));
+        R = held_done_ = upto;
+        if (!keep) held_ = false;
+      } else {
+        drop_held();
+      }
+    }
+    if (to <= R) return;
+    drop_held();
+    const uint64_t end = (next_to > to && next_to - to <= to - R) ? next_to : to;
+    round_launch(ctx_, g_, model_, seed_, id_base_ + R, end - R, id_base_, true, rd, stream_of(rd), false);
+    const bool keep = end > to;
+    account(round_finalize(ctx_, g_, rd, to - R, 0, keep));
+    if (keep) {
+      held_ = true;
+      held_first_ = R;
+      held_done_ = to;
+      held_end_ = end;
+    }
+    R = to;
+  }
+
+  // Discard the rest of a held launch (the loop stopped or moved on).
+  void drop_held() {
+    if (!held_) return;
+    Round& rd = ctx_->rounds[0];
+    rd.launched = false;
+    rd.waited = false;
+    held_ = false;
+  }
+
   void grow_elim(uint64_t& R, uint64_t to) {
     while (R < to) {
       const uint64_t need = to - R;
@@ -228,6 +281,8 @@ class RoundSampler {
   Exchange ex_;
   bool speculate_ = false;
   Round* spec_ = nullptr;
+  bool lookahead_ = false, held_ = false;
+  uint64_t held_first_ = 0, held_done_ = 0, held_end_ = 0;
 };
 
 }  // namespace

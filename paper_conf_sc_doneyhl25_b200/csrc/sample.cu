@@ -947,7 +947,8 @@ __global__ void compact_sizes_kernel(const uint32_t* __restrict__ sizes, const u
 // set index of sample s is set_index0 + kidx[s] (empty sets dropped).
 template <class GV>
 __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint64_t nslots,
-                               const uint64_t* __restrict__ set_start, uint64_t set_index0, uint32_t use,
+                               const uint64_t* __restrict__ set_start, uint64_t set_index0, uint32_t from,
+                               uint32_t use,
                                uint32_t* __restrict__ fill, uint32_t* __restrict__ arena, uint32_t ab,
                                uint32_t* __restrict__ C, GV g, bool ic, unsigned long long* __restrict__ esum,
                                const uint32_t* __restrict__ roots, const uint32_t* __restrict__ kidx) {
@@ -957,7 +958,7 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
     const unsigned long long k = keys[i];
     if (k == 0ull) continue;
     const uint32_t s_local = (uint32_t)(k >> 32) - 1u;
-    if (s_local >= use) continue;  // speculative samples beyond the ones kept
+    if (s_local >= use || s_local < from) continue;  // samples outside the appended range
     const uint32_t v = (uint32_t)k;
     if (ic) e += g_off(g, v + 1) - g_off(g, v);
     if (roots && v == roots[s_local]) continue;
@@ -1184,6 +1185,7 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
     EIM_CUDA(cudaMemsetAsync(rd.dbg.p, 0, 64 * count, st));
   }
   rd.nlaunch = 0;
+  rd.waited = false;
   round_kernel(ctx, g, rd, st, spare_sm_slot);
 }
 
@@ -1240,10 +1242,11 @@ void round_cancel(eim_ctx* ctx, Round& rd) {
   rd.qdirty = true;  // items may be left in the queue
 }
 
-SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use) {
+SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from, bool keep) {
   SampleResult res;
   if (!rd.launched || rd.count == 0) return res;
-  if (use > rd.count) fail(EIM_E_STATE, "round_finalize beyond the launched range");
+  if (use > rd.count || from > use) fail(EIM_E_STATE, "round_finalize beyond the launched range");
+  if (from > 0 && (rd.rflags & RF_DROP_ROOT)) fail(EIM_E_STATE, "partial appends of an eliminating round");
   cudaStream_t st = ctx->stream;
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
   SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
@@ -1255,7 +1258,7 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     }
     return (double)total;
   };
-  for (int attempt = 0;; ++attempt) {
+  for (int attempt = 0; !rd.waited; ++attempt) {
     int counted = 0;
     for (;;) {  // until every id is taken and no task is outstanding (a paused round is resumed here)
       EIM_CUDA(cudaStreamWaitEvent(st, rd.ev[2 * rd.nlaunch - 1], 0));
@@ -1293,17 +1296,22 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
       round_start(ctx, g, rd, st, false);
       continue;
     }
-    break;
+    rd.waited = true;
   }
-  rd.launched = false;
-  res.kept = res.consumed = use;
-  if (use == 0) return res;
+  // ---- append the sets of s_local in [from, use); with keep the round's
+  // table stays for a later append of the rest
+  if (!keep) {
+    rd.launched = false;
+    rd.waited = false;
+  }
+  res.kept = res.consumed = use - from;
+  if (use == from) return res;
   const bool drop_root = (rd.rflags & RF_DROP_ROOT) != 0;
   const bool drop_empty = drop_root && (rd.rflags & RF_DROP_EMPTY) != 0;
-  uint32_t* sizes = rd.sizes.as<uint32_t>();
+  uint32_t* sizes = rd.sizes.as<uint32_t>() + from;
   uint32_t* roots = nullptr;
   uint32_t* kidx = nullptr;
-  uint64_t consumed = use, nsets = use;
+  uint64_t consumed = use, nsets = use - from;
   size_t tmp = 0, tmp2 = 0;
   if (drop_root) {
     // ---- source elimination (R22): roots out of the sets; with drop_empty
@@ -1350,36 +1358,38 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     }
   }
   res.kept = nsets;
-  res.consumed = consumed;
+  res.consumed = consumed - from;
   // ---- sizes -> offsets (sample-id order) -> arena placement -> scatter + histogram
   uint64_t* excl = rd.excl.as<uint64_t>();
   const uint64_t set_index0 = rd.first - rd.set_base;
-  ensure_sets(ctx, set_index0 + std::max<uint64_t>(nsets, 1));
+  ensure_sets(ctx, set_index0 + from + std::max<uint64_t>(nsets, 1));
   sizes_to_offsets_kernel<<<grid_for(ctx, nsets + 1, 256), 256, 0, st>>>(sizes, nsets, excl);
   EIM_CUDA(cudaGetLastError());
   const bool ic = rd.model == EIM_IC;
   unsigned long long* d_edges_sum = &ctl->edges;  // IC: summed by the scatter; LT: reduced from per-walk steps
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, nsets + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, consumed, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>() + from, d_edges_sum,
+                                           consumed - from, st));
   ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, nsets + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>(), d_edges_sum, consumed, st));
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>() + from, d_edges_sum,
+                                           consumed - from, st));
   else EIM_CUDA(cudaMemsetAsync(d_edges_sum, 0, sizeof(unsigned long long), st));
   EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + nsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   const uint64_t total = h->ticket, cursor = ctx->arena_used;
   arena_ensure(ctx, cursor + total);
   if (nsets) {
-    place_sets_kernel<<<grid_for(ctx, nsets, 256), 256, 0, st>>>(excl, sizes, nsets, cursor, set_index0,
+    place_sets_kernel<<<grid_for(ctx, nsets, 256), 256, 0, st>>>(excl, sizes, nsets, cursor, set_index0 + from,
                                                                   ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>());
     EIM_CUDA(cudaGetLastError());
   }
-  EIM_CUDA(cudaMemsetAsync(rd.fill.p, 0, consumed * sizeof(uint32_t), st));
+  EIM_CUDA(cudaMemsetAsync(rd.fill.as<uint32_t>() + from, 0, (consumed - from) * sizeof(uint32_t), st));
   const uint64_t nslots = 1ull << rd.bits;
   auto scatter = [&](auto gv) {
     scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
         rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
-        (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
+        (uint32_t)from, (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
         rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_sum, roots, kidx);
   };
   if (g->packed) scatter(g->pview);
@@ -1391,7 +1401,7 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   res.edges = h->edges;
-  ctx->est_mean_size = std::max(1.0, (double)(total + (drop_root ? consumed : 0)) / (double)consumed);
+  ctx->est_mean_size = std::max(1.0, (double)(total + (drop_root ? consumed : 0)) / (double)(consumed - from));
   return res;
 }
 
