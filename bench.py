@@ -376,7 +376,7 @@ def main():
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": workload_desc(args.config), "theta": theta_all,
                        "parallelism": f"sample-range dp{world} (graph replicated)",
-                       "l2": "flushed between steps (256 MiB write); graph 315 MB > 126 MB L2"},
+                       "l2": f"flushed between steps (256 MiB write); graph {(off.nbytes + nbr.nbytes) / 1e6:.0f} MB > 126 MB L2"},
             "imm_s": ms_per_step / 1e3,
             "traversed_edges_per_s": float(edges.item()) / (ms * 1e-3) if world == 1 else float(edges.item()) / (float(t.item()) * 1e-3),
             "sampler_sets_per_s": theta_all / (sum(s["ms_sample"] for s in stats) / args.steps / 1e3),

@@ -251,11 +251,11 @@ eim_status eim_graph_free(eim_graph* g) {
     // every kernel that reads the graph has finished when a hot-path call
     // returns (the calls end synchronised), so the free is stream-ordered
     cudaSetDevice(ctx->device);
-    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum})
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum, g->d_aug})
       if (p) cudaFreeAsync(p, ctx->stream);
     cudaStreamSynchronize(ctx->stream);
   } else {
-    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum})
+    for (void* p : {g->d_off, g->d_nbr, g->d_thr, g->d_offw, g->d_nbrw, g->d_x, g->d_cum, g->d_aug})
       if (p) cudaFree(p);
   }
   g->magic = 0;

@@ -128,6 +128,8 @@ struct eim_graph {
   eim::WeightedGraphView wview{};
   void* d_x = nullptr;
   void* d_cum = nullptr;
+  void* d_aug = nullptr;         // LT walk store of the plain graph, built on the first LT run (uint4 per in-edge)
+  uint64_t aug_bytes = 0;
   bool lt_ok = true;             // weighted: every row's weights sum to <= 2^32 (LT usable)
   uint64_t bytes = 0;            // device bytes of the store
   int proper_edge = -1;  // has an edge u -> v, u != v (1/0; -1 = not yet computed)

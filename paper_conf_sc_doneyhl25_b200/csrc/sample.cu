@@ -882,6 +882,147 @@ __global__ void __launch_bounds__(256) lt_kernel(GV g, RoundView R, uint64_t cou
   if (edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
 
+// LT walk store of the plain graph: aug[e] = (v, d^-(v), lo32 off[v],
+// hi32 off[v]) for v = in_nbr[e].  One 16-byte load per walk step then gives
+// the chosen in-neighbour AND its row, so a step is one dependent memory
+// round trip (the row-offset load of v disappears from the critical path).
+// 16 B per in-edge (C3: 1.9 GB), built once per graph on the first LT run.
+__global__ void lt_aug_build_kernel(GraphView g, uint4* __restrict__ aug) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < g.m; e += stride) {
+    const uint32_t v = __ldg(g.nbr + e);
+    const uint64_t o0 = __ldg(g.off + v), o1 = __ldg(g.off + v + 1);
+    aug[e] = make_uint4(v, (uint32_t)(o1 - o0), (uint32_t)o0, (uint32_t)(o0 >> 32));
+  }
+}
+
+// A key of no sample (its sample field decodes to 0xFFFFFFFE, above every
+// round's count, so the scatter skips it): written over a speculative insert
+// that the walk turned out not to reach.
+constexpr unsigned long long TABLE_TOMB = 0xFFFFFFFF00000000ull;
+
+// Second half of table_insert, for a first CAS issued earlier at slot i
+// whose result is cur: 1 = inserted (*slot = its slot), 0 = present, -1 =
+// table too full (same probe budget as table_insert).
+__device__ __forceinline__ int table_resolve(unsigned long long* keys, uint32_t bits, unsigned long long key,
+                                             uint32_t i, unsigned long long cur, uint32_t* slot) {
+  const uint32_t mask = (uint32_t)((1ull << bits) - 1ull);
+  for (uint32_t p = 1;; ++p) {
+    if (cur == 0ull) {
+      *slot = i;
+      return 1;
+    }
+    if (cur == key) return 0;
+    if (p == MAX_PROBE) return -1;
+    i = (i + 1u) & mask;
+    cur = atomicCAS(&keys[i], 0ull, key);
+  }
+}
+
+// lt_kernel on the walk store (same walk, same draws, same outputs).  The
+// walk runs one step ahead of its stop test: the membership insert of the
+// next vertex and the load of the entry after it are issued before the
+// insert of the current vertex is resolved, so a step costs one memory round
+// trip.  When the current vertex turns out to be a revisit (the walk stops,
+// P:136), the speculative insert is overwritten with TABLE_TOMB.
+__global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* __restrict__ aug, RoundView R,
+                                                     uint64_t count, SampleCtl* ctl) {
+  const PhiloxKey& K = R.K;
+  unsigned long long edges_acc = 0;
+  for (;;) {
+    const volatile unsigned int* cp = R.cancel;
+    if (cp[0] || cp[1]) break;  // cancelled or paused
+    const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
+    if (t >= count) break;
+    const uint32_t s_local = (uint32_t)t;
+    const uint64_t s = R.base + s_local;
+    const uint32_t u = draw_root(s, g.n, K);
+    const uint64_t e0 = __ldg(g.off + u);
+    const uint32_t d = (uint32_t)(__ldg(g.off + u + 1) - e0);
+    const uint32_t tau = word_of(philox_at((uint64_t)(u >> 2), s, TAG_LT, K), u & 3u);
+    bool ok = table_insert(R.keys, R.bits, table_key(s_local, u)) >= 0;
+    uint32_t L = 1;
+    unsigned long long steps = 0;
+    if (ok && d) {
+      // the step from the root: entry a -> vertex v (insert pending), nx = the entry chosen from v
+      const uint4 a = __ldg(aug + e0 + __umul64hi((unsigned long long)tau << 32, d));
+      steps = 1;
+      uint32_t v = a.x;
+      unsigned long long key = table_key(s_local, v);
+      uint32_t slot = table_hash(key, R.bits);
+      unsigned long long cur = atomicCAS(&R.keys[slot], 0ull, key);
+      bool nxt = a.y != 0u;
+      uint4 nx = a;
+      if (nxt) {
+        const uint32_t tv = word_of(philox_at((uint64_t)(v >> 2), s, TAG_LT, K), v & 3u);
+        nx = __ldg(aug + ((uint64_t)a.z | ((uint64_t)a.w << 32)) + __umul64hi((unsigned long long)tv << 32, a.y));
+      }
+      for (;;) {
+        // speculate the step from v: v2 = nx.x, its insert and the entry chosen from v2
+        uint32_t v2 = 0, slot2 = 0;
+        unsigned long long key2 = 0, cur2 = 0;
+        bool nxt2 = false;
+        uint4 nx2 = nx;
+        if (nxt) {
+          v2 = nx.x;
+          key2 = table_key(s_local, v2);
+          slot2 = table_hash(key2, R.bits);
+          cur2 = atomicCAS(&R.keys[slot2], 0ull, key2);
+          nxt2 = nx.y != 0u;
+          if (nxt2) {
+            const uint32_t tv2 = word_of(philox_at((uint64_t)(v2 >> 2), s, TAG_LT, K), v2 & 3u);
+            nx2 = __ldg(aug + ((uint64_t)nx.z | ((uint64_t)nx.w << 32)) + __umul64hi((unsigned long long)tv2 << 32, nx.y));
+          }
+        }
+        // resolve v's insert
+        uint32_t got = 0;
+        const int ins = table_resolve(R.keys, R.bits, key, slot, cur, &got);
+        if (ins <= 0) {
+          if (ins < 0) ok = false;
+          // v was a revisit (or the table is full): undo v2's insert if it landed
+          if (nxt) {
+            uint32_t got2 = 0;
+            if (table_resolve(R.keys, R.bits, key2, slot2, cur2, &got2) > 0) R.keys[got2] = TABLE_TOMB;
+          }
+          break;
+        }
+        ++L;
+        if (!nxt) break;  // d^-(v) = 0
+        ++steps;          // the step from v is real
+        v = v2;
+        key = key2;
+        slot = slot2;
+        cur = cur2;
+        nxt = nxt2;
+        nx = nx2;
+      }
+    }
+    if (ok) {
+      R.sizes[s_local] = L;
+      R.edges[s_local] = steps;
+      edges_acc += steps;
+    } else {
+      atomicOr(reinterpret_cast<unsigned int*>(&ctl->arena_fail), 1u);
+    }
+  }
+  if (edges_acc) atomicAdd(&ctl->edges, edges_acc);
+}
+
+static const uint4* lt_aug(eim_ctx* ctx, const eim_graph* gc, cudaStream_t st) {
+  if (std::getenv("EIM_NO_LT_AUG") || gc->packed || gc->weighted) return nullptr;
+  eim_graph* g = const_cast<eim_graph*>(gc);  // lazily built cache of the (immutable) store
+  if (!g->d_aug) {
+    const uint64_t bytes = std::max<uint64_t>(g->view.m, 1) * sizeof(uint4);
+    EIM_CUDA(cudaMallocAsync(&g->d_aug, bytes, st));
+    lt_aug_build_kernel<<<grid_for(ctx, g->view.m, 256), 256, 0, st>>>(g->view, static_cast<uint4*>(g->d_aug));
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches++;
+    g->aug_bytes = bytes;
+    g->bytes += bytes;
+  }
+  return static_cast<const uint4*>(g->d_aug);
+}
+
 // ---------------------------------------------------------------- output
 __global__ void sizes_to_offsets_kernel(const uint32_t* __restrict__ sizes, uint64_t count,
                                         uint64_t* __restrict__ out) {
@@ -1130,6 +1271,7 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
   if (rd.nlaunch >= Round::MAX_LAUNCH) fail(EIM_E_STATE, "too many sampler launches in one round");
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
   const RoundView R = round_view(rd);
+  const uint4* aug = rd.model == EIM_IC ? nullptr : lt_aug(ctx, g, st);  // built outside the launch's events
   EIM_CUDA(cudaEventRecord(rd.ev[2 * rd.nlaunch], st));
   if (rd.model == EIM_IC) {
     launch_ic<IC_G, IC_NSG>(ctx, g, R, rd.count, ctl, st, spare_sm_slot);
@@ -1139,7 +1281,8 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
     if (spare_sm_slot && per_sm > 1) per_sm -= 1;
     uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
     const uint32_t grid = (uint32_t)std::max<uint64_t>(blocks, 1);
-    if (g->packed) lt_kernel<<<grid, 256, 0, st>>>(g->pview, R, rd.count, ctl);
+    if (aug) lt_aug_kernel<<<grid, 256, 0, st>>>(g->view, aug, R, rd.count, ctl);
+    else if (g->packed) lt_kernel<<<grid, 256, 0, st>>>(g->pview, R, rd.count, ctl);
     else if (g->weighted) lt_kernel<<<grid, 256, 0, st>>>(g->wview, R, rd.count, ctl);
     else lt_kernel<<<grid, 256, 0, st>>>(g->view, R, rd.count, ctl);
     EIM_CUDA(cudaGetLastError());
