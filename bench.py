@@ -23,6 +23,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+LT_STEP_BYTES = 24.0  # LT walk step on the walk store: 16-B entry + 8-B table key
 METRIC = "RRR sets/s, traversed edges/s, end-to-end IMM s (k=50, eps=0.5) at 1/2/4/8 B200"
 UNIT = "RRR sets/s"
 GRAPH_SEED = 1
@@ -249,11 +250,11 @@ def main():
         peak, peak_src = philox_roof_gwords() if rank == 0 else (1630.0, "")
         achieved = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
     else:
-        # LT walk step: in_off pair (16 B) + the chosen in_nbr (4 B) + one
-        # 8-B membership-table key = 28 algorithmic bytes
+        # LT walk step on the walk store: one 16-B entry (v, d(v), off[v]) + one
+        # 8-B membership-table key = 24 algorithmic bytes
         peak = float(_peaks().get("hbm_gbs", 8000.0))
         peak_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in _peaks() else "fallback 8 TB/s"
-        achieved = (28.0 * k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
+        achieved = (LT_STEP_BYTES * k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
     traffic = None  # DRAM bytes per sampler launch from the committed ncu --set full capture
     tpath = os.path.join(ROOT, "profiles", "ncu_sampler.json" if c["model"] == "IC" else "ncu_sampler_lt.json")
     if os.path.exists(tpath):
@@ -390,14 +391,14 @@ def main():
                           "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge; best of the "
                                         "plain and the sampler's hoisted form, tools/philox_roof), "
                                         + peak_src + "; DESIGN.md §6"} if c["model"] == "IC" else
-                         {"bound": "hbm", "kernel": "lt_kernel (LT reverse walks)", "achieved": achieved,
+                         {"bound": "hbm", "kernel": "lt_aug_kernel (LT reverse walks on the walk store)", "achieved": achieved,
                           "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
                           "traffic": traffic,
-                          "peak_basis": "28 algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
-            # IC: examined edges/s vs the Philox roof; LT: 28 algorithmic bytes per walk step vs HBM
+                          "peak_basis": f"{LT_STEP_BYTES:.0f} algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
+            # IC: examined edges/s vs the Philox roof; LT: LT_STEP_BYTES per walk step vs HBM
             "sampler_fixed_budget": (dict(budget, frac=(budget["edges_per_s"] / 1e9 / world / peak)
                                           if c["model"] == "IC" else
-                                          (28.0 * budget["edges_per_s"] / 1e9 / world / peak))
+                                          (LT_STEP_BYTES * budget["edges_per_s"] / 1e9 / world / peak))
                                      if budget else None),
             "cpu_baseline": cb,
             "e2e": {"value": theta_all / (e2e_ms_step / 1e3), "unit": UNIT,
