@@ -484,3 +484,23 @@ def test_task_pool_layout_change_between_rounds(eim, ctx, graphs, monkeypatch):
         _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 20000, 1000)
     finally:
         eim.eim_graph_free(g)
+
+
+# LT walk store (lt_aug_kernel, default on the plain store) and the
+# row-offset walk (lt_kernel, EIM_NO_LT_AUG=1) against the oracle.  Cycles
+# make every walk end at a revisit (the speculative insert past it is
+# tombstoned), bigcycle gives 3000-step walks, the path graph ends walks at
+# d = 0, dense R-MAT mixes both; the same graph object serves both switches.
+@pytest.mark.parametrize("store", ["walk_store", "row_offsets"])
+def test_lt_walk_store_vs_row_offsets(eim, ctx, graphs, store, monkeypatch):
+    if store == "row_offsets":
+        monkeypatch.setenv("EIM_NO_LT_AUG", "1")
+    cases = [inputs.cycle_graph(40), inputs.cycle_graph(3000), inputs.path_graph(500),
+             inputs.rmat(600, 60000, seed=4), graphs("C1")]
+    for off, nbr in cases:
+        g = eim.eim_load_graph_csr(ctx, off, nbr)
+        try:
+            _sets_equal(eim, ctx, g, off, nbr, "LT", 5, 0, 1500)
+            _sets_equal(eim, ctx, g, off, nbr, "LT", 5, 2**40 + 7, 257)
+        finally:
+            eim.eim_graph_free(g)
