@@ -88,6 +88,7 @@ def _load():
             "orc_sample_ex": (ctypes.POINTER(_Arena), [U32, P, P, I32, U64, U64, U64, U32, I32]),
             "orc_arena_free": (None, [ctypes.POINTER(_Arena)]),
             "orc_greedy": (U64, [U32, U64, P, P, U32, P, P]),
+            "orc_coverage": (None, [U32, U64, P, P, P]),
             "orc_imm_params": (I32, [U32, U32, D, D, ctypes.POINTER(Params)]),
             "orc_imm": (I32, [U32, P, P, U32, D, D, I32, U64, I32, P, P, P, ctypes.POINTER(ImmStats)]),
             "orc_imm_ex": (I32, [U32, P, P, U32, D, D, I32, U64, U32, I32, P, P, P, ctypes.POINTER(ImmStats)]),
@@ -200,6 +201,17 @@ def greedy(n, offsets, members, k):
     gains = np.zeros(k, dtype=np.uint64)
     cov = _load().orc_greedy(n, offsets.size - 1, _ptr(offsets), _ptr(members), k, _ptr(seeds), _ptr(gains))
     return seeds, gains, int(cov)
+
+
+def coverage(n, offsets, members):
+    """C u32[n]: number of sets containing each vertex."""
+    offsets = np.ascontiguousarray(offsets, dtype=np.uint64)
+    members = np.ascontiguousarray(members, dtype=np.uint32)
+    if members.size == 0:
+        members = np.zeros(1, dtype=np.uint32)
+    C = np.zeros(n, dtype=np.uint32)
+    _load().orc_coverage(n, offsets.size - 1, _ptr(offsets), _ptr(members), _ptr(C))
+    return C
 
 
 def imm_params(n, k, eps, ell):

@@ -17,6 +17,8 @@
  *   orc_lt_choice ...... pinned (closed form floor(tau*d), exhaustive bounds)
  *   orc_rrr_set ........ pinned (materialised live-edge world + library BFS;
  *                        exact enumeration of worlds, RIS unbiasedness)
+ *   orc_coverage ....... pinned (closed forms: path/cycle/empty graph,
+ *                        sum = arena size, brute-force membership count)
  *   orc_greedy ......... pinned (brute force OPT, (1-1/e) bound, marginal
  *                        gains, tie order)
  *   orc_imm_params ..... pinned (mpmath 40-digit evaluation of [22] Eq. 6/9)
@@ -97,6 +99,9 @@ void       orc_arena_free(orc_arena* a);
 /* returns cov = sum of gains */
 uint64_t orc_greedy(uint32_t n, uint64_t num_sets, const uint64_t* offsets, const uint32_t* members,
                     uint32_t k, uint32_t* seeds_out, uint64_t* gains_out);
+
+/* coverage counts C[v] = #sets containing v (Alg. 2 l.25) */
+void orc_coverage(uint32_t n, uint64_t num_sets, const uint64_t* offsets, const uint32_t* members, uint32_t* C);
 
 /* ---- IMM (Alg. 1; [22] Alg. 1-3, Eq. 6 and 9) --------------- */
 typedef struct {

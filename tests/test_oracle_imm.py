@@ -122,3 +122,108 @@ def test_invalid_parameters():
                  (10, 2, 1.0, 1.0), (10, 2, 0.5, 0.0)]:
         with pytest.raises(ValueError):
             oracle.imm_params(*args)
+
+
+# ---------------------------------------------------------------- closed forms
+# The stop test, LB and theta of the martingale loop ([22] Alg. 2; prose at
+# P:65 and P:76) pinned on graphs where one vertex lies in EVERY RRR set
+# (path 0 -> 1 -> ..., hub -> leaves, directed cycle; in-degree <= 1 means
+# p = 1 under WC, so IC and LT sets are the same deterministic sets): the
+# first greedy pick covers all of R, so cov_i = |R| = theta_i in every round
+# and the stop test cov_i 2^i >= (1+eps') |R| reduces to 2^i >= 1+eps'.  The
+# loop therefore breaks at the first i >= 1 with 2^i >= 1+eps' (i = 1 when
+# eps <= 1/sqrt 2, else i = 2), provided i < log2 n; then LB = n / (1+eps')
+# and theta = max(theta_i, ceil(lambda* (1+eps') / n)).  If the loop runs out
+# (i < log2 n fails first) LB = 1 and theta = max(theta_last, ceil(lambda*)).
+# Everything below is evaluated in mpmath at 40 digits, independently of the
+# oracle's double arithmetic; a wrong comparison (> vs >=, <= log2 n), a wrong
+# LB or theta_i instead of |R| changes one of the integers.
+def _mp_ceil_safe(x):
+    c = mpmath.ceil(x)
+    assert c - x > mpmath.mpf("1e-9") or x == c, f"knife edge for ceil: {x}"
+    return int(c)
+
+
+def closed_form_all_covered(n, k, eps, ell):
+    mp = _mp_params(n, k, eps, ell)
+    log2n = mpmath.log(n, 2)
+    thetas, lb, i = [], None, 1
+    while i < log2n:
+        thetas.append(_mp_ceil_safe(mp["lambda_p"] * 2**i / n))
+        if 2**i >= 1 + mp["eps_p"]:
+            lb = n / (1 + mp["eps_p"])
+            break
+        i += 1
+    theta = max(thetas[-1] if thetas else 0, _mp_ceil_safe(mp["lambda_s"] / (lb if lb is not None else 1)))
+    return dict(theta_i=thetas, lb=lb, theta=theta)
+
+
+ALL_COVERED_GRAPHS = {"path": inputs.path_graph, "star": inputs.star_out, "cycle": inputs.cycle_graph}
+ALL_COVERED_CASES = [  # (n, k, eps, ell): i* = 1 / i* = 2 / loop bound hit / no round at all
+    (33, 1, 0.5, 1.0), (33, 3, 0.9, 1.0), (1000, 2, 0.1, 2.0), (5, 2, 0.9, 1.0), (4, 1, 0.9, 1.0),
+    (4, 2, 0.5, 1.0), (2, 1, 0.3, 1.0), (300, 5, 0.69, 0.5), (300, 5, 0.72, 0.5)]
+
+
+@pytest.mark.parametrize("shape", sorted(ALL_COVERED_GRAPHS))
+@pytest.mark.parametrize("model", ["IC", "LT"])
+@pytest.mark.parametrize("n,k,eps,ell", ALL_COVERED_CASES)
+def test_imm_stop_test_lb_theta_closed_form(shape, model, n, k, eps, ell):
+    off, nbr = ALL_COVERED_GRAPHS[shape](n)
+    want = closed_form_all_covered(n, k, eps, ell)
+    r = oracle.imm(off, nbr, k, eps, ell, model, 11)
+    assert r["theta_i"] == want["theta_i"]
+    assert r["cov_i"] == want["theta_i"]        # the first pick covers every set
+    assert r["rounds"] == len(want["theta_i"])
+    if want["lb"] is None:
+        assert r["lb"] == 1.0
+    else:
+        assert abs(r["lb"] - float(want["lb"])) <= 1e-12 * float(want["lb"])
+    assert r["theta"] == want["theta"]
+    assert r["cov"] == r["theta"] and r["spread"] == float(n)
+    # vertex 0 first; every later pick has gain 0 and is the lowest unselected id (R10)
+    assert r["seeds"].tolist() == list(range(k))
+
+
+def test_closed_form_reaches_both_break_rounds():
+    # the case table exercises a break at i = 1, a break at i = 2, the loop
+    # bound (i < log2 n) and the empty loop -- keep it that way
+    kinds = set()
+    for n, k, eps, ell in ALL_COVERED_CASES:
+        w = closed_form_all_covered(n, k, eps, ell)
+        kinds.add((len(w["theta_i"]), w["lb"] is None))
+    assert {(1, False), (2, False), (1, True), (0, True)} <= kinds
+
+
+# Coverage counts C[v] = #sets containing v (Alg. 2 l.25).
+def test_coverage_closed_forms():
+    n, cnt = 40, 3000
+    for model in ("IC", "LT"):
+        # path 0 -> ... -> n-1 with p = 1: RR(root) = {0..root}, so C[j] = #{s : root_s >= j}
+        off, nbr = inputs.path_graph(n)
+        o, m, _ = oracle.sample(off, nbr, model, 3, 0, cnt)
+        roots = np.array([oracle.root(3, s, n) for s in range(cnt)])
+        want = np.array([(roots >= j).sum() for j in range(n)])
+        assert np.array_equal(oracle.coverage(n, o, m), want)
+        # cycle: every set is V
+        off, nbr = inputs.cycle_graph(n)
+        o, m, _ = oracle.sample(off, nbr, model, 3, 0, cnt)
+        assert np.array_equal(oracle.coverage(n, o, m), np.full(n, cnt))
+    # no edges: singleton sets, C = root frequencies
+    off, nbr = inputs.empty_graph(n)
+    o, m, _ = oracle.sample(off, nbr, "IC", 4, 0, cnt)
+    roots = [oracle.root(4, s, n) for s in range(cnt)]
+    assert np.array_equal(oracle.coverage(n, o, m), np.bincount(roots, minlength=n))
+
+
+def test_coverage_brute_force_random_arenas():
+    rng = np.random.default_rng(5)
+    for _ in range(20):
+        n = int(rng.integers(1, 60))
+        sets = [rng.choice(n, size=int(rng.integers(0, n + 1)), replace=False) for _ in range(int(rng.integers(0, 40)))]
+        offs = np.zeros(len(sets) + 1, dtype=np.uint64)
+        offs[1:] = np.cumsum([len(s) for s in sets])
+        mem = np.concatenate(sets).astype(np.uint32) if sets and offs[-1] else np.zeros(0, dtype=np.uint32)
+        C = oracle.coverage(n, offs, mem)
+        for v in range(n):
+            assert C[v] == sum(1 for s in sets if v in set(s.tolist()))
+        assert int(C.sum()) == int(offs[-1])
