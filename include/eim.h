@@ -230,6 +230,18 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
                             const uint32_t* members, uint32_t k, uint32_t* seeds_out,
                             uint64_t* gains_out);
 
+/* eim_get_coverage: the coverage counts C[v] = number of RRR sets of R that
+ * contain v ("counts the occurrences of each vertex across all RRR
+ * sets"; Alg. 2 l.25), for the R of the most recent eim_imm_run /
+ * eim_imm_run_ex (the final R, theta sets; the fresh sets with
+ * EIM_F_FRESH_FINAL) or eim_select_seeds (the given arena) on ctx.  These are
+ * the counts the first greedy pick of the final NodeSelection maximises.
+ * C_out[n] is a caller-allocated host buffer; n must equal the vertex count
+ * of that call.  Errors: EIM_E_STATE (no such call on ctx yet, or the last
+ * hot-path call was eim_sample_rrr, which builds no counts), EIM_E_INVAL
+ * (C_out NULL or n different), EIM_E_CUDA. */
+eim_status eim_get_coverage(eim_ctx* ctx, uint32_t n, uint32_t* C_out);
+
 /* Statistics of the most recent eim_imm_run / eim_sample_rrr call on ctx
  * (for eim_sample_rrr: theta = count, edges_examined, sample_launches,
  * spilled_samples, ms_sample_kernel, ms_sample, ms_total, arena_elems,

@@ -55,14 +55,13 @@ static void* gen_worker(void* arg) {
   j->oom = 0;
   for (uint64_t t = j->t0; t < j->t1; ++t) {
     uint32_t src = 0, dst = 0;
+    uint64_t r64 = 0;
     for (uint32_t lvl = 0; lvl < j->s; ++lvl) {
-      uint64_t r64 = rnd(j->seed_h, t, lvl >> 1);
+      if ((lvl & 1) == 0) r64 = rnd(j->seed_h, t, lvl >> 1);  /* one 64-bit word per two levels */
       uint32_t r = (lvl & 1) ? (uint32_t)(r64 >> 32) : (uint32_t)r64;
-      uint32_t sb, db;
-      if (r < j->ta) { sb = 0; db = 0; }
-      else if (r < j->tab) { sb = 0; db = 1; }
-      else if (r < j->tabc) { sb = 1; db = 0; }
-      else { sb = 1; db = 1; }
+      /* quadrant: [0,ta) -> (0,0), [ta,tab) -> (0,1), [tab,tabc) -> (1,0), else (1,1) */
+      const uint32_t ga = r >= j->ta, gb = r >= j->tab, gc = r >= j->tabc;
+      const uint32_t sb = gb, db = ga ^ gb ^ gc;
       src = (src << 1) | sb;
       dst = (dst << 1) | db;
     }
@@ -84,17 +83,15 @@ static void* gen_worker(void* arg) {
   return NULL;
 }
 
-/* stable LSD radix sort of (key, idx) by key */
-static int radix_sort(uint64_t* keys, uint64_t* idx, uint64_t N, int key_bits) {
-  uint64_t* k2 = (uint64_t*)malloc((N ? N : 1) * sizeof(uint64_t));
-  uint64_t* i2 = (uint64_t*)malloc((N ? N : 1) * sizeof(uint64_t));
-  if (!k2 || !i2) { free(k2); free(i2); return -1; }
+/* stable LSD radix sort of (key, idx) by key over [0, N) (single thread);
+ * k2/i2 are scratch of N entries; the result ends in keys/idx. */
+static void lsd_sort(uint64_t* keys, uint64_t* idx, uint64_t* k2, uint64_t* i2, uint64_t N, int key_bits) {
   const int DB = 11;
   const uint64_t NB = 1u << DB;
-  uint64_t* cnt = (uint64_t*)malloc(NB * sizeof(uint64_t));
+  uint64_t cnt[1u << 11];
   uint64_t *ka = keys, *ia = idx, *kb = k2, *ib = i2;
   for (int shift = 0; shift < key_bits; shift += DB) {
-    memset(cnt, 0, NB * sizeof(uint64_t));
+    memset(cnt, 0, sizeof(cnt));
     for (uint64_t i = 0; i < N; ++i) cnt[(ka[i] >> shift) & (NB - 1)]++;
     uint64_t sum = 0;
     for (uint64_t b = 0; b < NB; ++b) { uint64_t c = cnt[b]; cnt[b] = sum; sum += c; }
@@ -111,7 +108,87 @@ static int radix_sort(uint64_t* keys, uint64_t* idx, uint64_t N, int key_bits) {
     memcpy(keys, ka, N * sizeof(uint64_t));
     memcpy(idx, ia, N * sizeof(uint64_t));
   }
-  free(k2); free(i2); free(cnt);
+}
+
+/* Parallel stable sort of (key, idx) by key: a stable partition on the top
+ * PB key bits (per-thread counts over contiguous chunks, chunk order kept),
+ * then every bucket LSD-sorted on the remaining bits by a pool of threads.
+ * Equal keys keep their input order, exactly as a sequential stable sort. */
+typedef struct {
+  uint64_t *keys, *idx, *k2, *i2;
+  uint64_t N, lo, hi;
+  int T, t, key_bits, low_bits, PB;
+  uint64_t* cnt;              /* T x NBK */
+  uint64_t* bstart;           /* NBK + 1 */
+  volatile uint64_t* next_b;  /* bucket claim counter (phase 3) */
+  pthread_mutex_t* mu;
+  int phase;
+} sort_job;
+
+static void* sort_worker(void* arg) {
+  sort_job* j = (sort_job*)arg;
+  const uint64_t NBK = 1ull << j->PB;
+  uint64_t* c = j->cnt + (uint64_t)j->t * NBK;
+  if (j->phase == 1) {
+    for (uint64_t i = j->lo; i < j->hi; ++i) c[j->keys[i] >> j->low_bits]++;
+  } else if (j->phase == 2) {
+    for (uint64_t i = j->lo; i < j->hi; ++i) {
+      uint64_t p = c[j->keys[i] >> j->low_bits]++;
+      j->k2[p] = j->keys[i];
+      j->i2[p] = j->idx[i];
+    }
+  } else {
+    for (;;) {
+      pthread_mutex_lock(j->mu);
+      uint64_t b = (*j->next_b)++;
+      pthread_mutex_unlock(j->mu);
+      if (b >= NBK) break;
+      uint64_t a = j->bstart[b], e = j->bstart[b + 1];
+      /* bucket data is in k2/i2; sort it there with keys/idx as scratch */
+      if (e > a) lsd_sort(j->k2 + a, j->i2 + a, j->keys + a, j->idx + a, e - a, j->low_bits);
+    }
+  }
+  return NULL;
+}
+
+static int radix_sort(uint64_t* keys, uint64_t* idx, uint64_t N, int key_bits, int T) {
+  uint64_t* k2 = (uint64_t*)malloc((N ? N : 1) * sizeof(uint64_t));
+  uint64_t* i2 = (uint64_t*)malloc((N ? N : 1) * sizeof(uint64_t));
+  if (!k2 || !i2) { free(k2); free(i2); return -1; }
+  if (T < 1) T = 1;
+  const int PB = key_bits < 11 ? key_bits : 11;
+  const uint64_t NBK = 1ull << PB;
+  uint64_t* cnt = (uint64_t*)calloc((size_t)T * NBK, sizeof(uint64_t));
+  uint64_t* bstart = (uint64_t*)calloc(NBK + 1, sizeof(uint64_t));
+  sort_job* jobs = (sort_job*)calloc((size_t)T, sizeof(sort_job));
+  pthread_t* th = (pthread_t*)calloc((size_t)T, sizeof(pthread_t));
+  pthread_mutex_t mu = PTHREAD_MUTEX_INITIALIZER;
+  volatile uint64_t next_b = 0;
+  if (!cnt || !bstart || !jobs || !th) { free(k2); free(i2); free(cnt); free(bstart); free(jobs); free(th); return -1; }
+  for (int phase = 1; phase <= 3; ++phase) {
+    if (phase == 2) {  /* exclusive offsets: bucket-major, thread (= chunk) order within a bucket */
+      uint64_t sum = 0;
+      for (uint64_t b = 0; b < NBK; ++b) {
+        bstart[b] = sum;
+        for (int t = 0; t < T; ++t) { uint64_t c = cnt[(uint64_t)t * NBK + b]; cnt[(uint64_t)t * NBK + b] = sum; sum += c; }
+      }
+      bstart[NBK] = sum;
+    }
+    for (int t = 0; t < T; ++t) {
+      sort_job* j = &jobs[t];
+      j->keys = keys; j->idx = idx; j->k2 = k2; j->i2 = i2; j->N = N;
+      j->lo = N * (uint64_t)t / (uint64_t)T;
+      j->hi = N * (uint64_t)(t + 1) / (uint64_t)T;
+      j->T = T; j->t = t; j->key_bits = key_bits; j->low_bits = key_bits - PB; j->PB = PB;
+      j->cnt = cnt; j->bstart = bstart; j->next_b = &next_b; j->mu = &mu; j->phase = phase;
+      pthread_create(&th[t], NULL, sort_worker, j);
+    }
+    for (int t = 0; t < T; ++t) pthread_join(th[t], NULL);
+  }
+  /* sorted data is in k2/i2 */
+  memcpy(keys, k2, N * sizeof(uint64_t));
+  memcpy(idx, i2, N * sizeof(uint64_t));
+  free(k2); free(i2); free(cnt); free(bstart); free(jobs); free(th);
   return 0;
 }
 
@@ -207,7 +284,7 @@ int rmat_generate(uint32_t n, uint64_t m, double a, double b, double c, uint64_t
       free(jobs[t].keys); free(jobs[t].idx);
     }
     free(jobs); free(th);
-    if (radix_sort(keys, idx, total, 32 + (int)s) != 0) return -1;
+    if (radix_sort(keys, idx, total, 32 + (int)s, nthreads) != 0) return -1;
     /* unique keys, keeping the first attempt (stable sort => smallest idx first) */
     uint64_t u = 0;
     for (uint64_t i = 0; i < total; ++i) {

@@ -33,7 +33,7 @@ EXPORTS = ["eim_create", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "ei
            "eim_load_graph_csr", "eim_load_graph_csr_ex", "eim_load_graph_csr_weighted", "eim_graph_bytes",
            "eim_graph_free", "eim_imm_run", "eim_imm_run_ex", "eim_sample_rrr",
            "eim_sample_rrr_ex", "eim_select_seeds",
-           "eim_imm_params", "eim_shard_range", "eim_get_stats"]
+           "eim_imm_params", "eim_shard_range", "eim_get_stats", "eim_get_coverage"]
 
 
 class EimError(RuntimeError):
@@ -110,6 +110,7 @@ def lib():
         "eim_imm_params": (_I, [_U32, _U32, _D, _D, ctypes.POINTER(ImmParams)]),
         "eim_shard_range": (_I, [_U64, _U64, _I, _I, ctypes.POINTER(_U64), ctypes.POINTER(_U64)]),
         "eim_get_stats": (_I, [_P, _P]),
+        "eim_get_coverage": (_I, [_P, _U32, _P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -247,6 +248,13 @@ def eim_get_stats(ctx):
     st = Stats()
     _check(lib().eim_get_stats(ctx, ctypes.addressof(st)), ctx)
     return st.as_dict()
+
+
+def eim_get_coverage(ctx, n):
+    """Coverage counts C u32[n] of the R of the last eim_imm_run / eim_select_seeds."""
+    C = np.zeros(n, dtype=np.uint32)
+    _check(lib().eim_get_coverage(ctx, n, C.ctypes.data), ctx)
+    return C
 
 
 # ------------------------------------------------------------------ host-only

@@ -294,7 +294,9 @@ eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double e
     if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
     if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
     if (model == EIM_LT && !g->lt_ok) fail(EIM_E_INVAL, "LT: a row's edge weights sum to more than 1");
+    ctx->cov_n = 0;
     imm_run(ctx, g, k, eps, ell, model, seed, flags, seeds_out, theta_out, spread_out, &ctx->last_stats);
+    ctx->cov_n = g->view.n;
     if (stats_out) *stats_out = ctx->last_stats;
   });
 }
@@ -321,6 +323,7 @@ eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, 
     cudaStream_t st = ctx->stream;
     const auto t0 = std::chrono::steady_clock::now();
     const uint64_t launches0 = ctx->kernel_launches;
+    ctx->cov_n = 0;
     arena_reset(ctx, g->packed ? bit_width((uint64_t)g->view.n - 1) : 32u);
     const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false,
                                         (flags & EIM_F_SOURCE_ELIM) ? RF_DROP_ROOT : 0u);
@@ -370,6 +373,7 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     for (uint64_t i = 0; i < total; ++i)
       if (members[i] >= n) fail(EIM_E_INVAL, "member id >= n");
     cudaStream_t st = ctx->stream;
+    ctx->cov_n = 0;
     arena_reset(ctx);
     ctx->stage_a.reserve((num_sets + 1) * sizeof(uint64_t), false, st);
     ctx->stage_b.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
@@ -386,6 +390,19 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     ctx->last_stats.theta = num_sets;
     ctx->last_stats.arena_elems = total;
     ctx->last_stats.ms_select = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    ctx->cov_n = n;
+  });
+}
+
+eim_status eim_get_coverage(eim_ctx* ctx, uint32_t n, uint32_t* C_out) {
+  if (!ctx_ok(ctx)) return EIM_E_STATE;
+  return guarded(ctx, [&] {
+    if (ctx->cov_n == 0) fail(EIM_E_STATE, "no coverage counts: run eim_imm_run or eim_select_seeds first");
+    if (!C_out) fail(EIM_E_INVAL, "C_out is NULL");
+    if (n != ctx->cov_n) fail(EIM_E_INVAL, "n differs from the vertex count of the last call");
+    EIM_CUDA(cudaMemcpyAsync(C_out, ctx->C_total.p, (uint64_t)n * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                             ctx->stream));
+    EIM_CUDA(cudaStreamSynchronize(ctx->stream));
   });
 }
 

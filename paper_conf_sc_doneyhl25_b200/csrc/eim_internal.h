@@ -163,6 +163,7 @@ struct eim_ctx {
   void* h_pinned = nullptr;   // small pinned host scratch
   cudaEvent_t ev0, ev1;
   eim_stats last_stats;       // statistics of the most recent hot-path call
+  uint32_t cov_n = 0;         // n of the coverage counts C_total of the last imm_run / select_seeds (0: none)
 };
 
 namespace eim {

@@ -202,13 +202,42 @@ def test_invalid_graphs_rejected(eim, ctx):
 
 
 # ---------------------------------------------------------------- full size
-def test_C2_sampled_sets_and_imm(eim, ctx, graphs, monkeypatch):
+def _coverage_equal(eim, ctx, n, ro, rm):
+    """C after the last eim_imm_run == the oracle's counts over the same R."""
+    C = eim.eim_get_coverage(ctx, n)
+    assert np.array_equal(C, oracle.coverage(n, ro, rm))
+    return C
+
+
+def _exhaustive(eim, ctx, g, off, nbr, model, seed, theta, chunk=1 << 15):
+    """Every set of ids [0, theta) against the oracle (in chunks); returns the oracle arena."""
+    ro_all, rm_all = [np.zeros(1, dtype=np.uint64)], []
+    base = 0
+    for first in range(0, theta, chunk):
+        cnt = min(chunk, theta - first)
+        ro = _sets_equal(eim, ctx, g, off, nbr, model, seed, first, cnt)
+        ro_all.append(ro[1:] + np.uint64(base))
+        base += int(ro[-1])
+    ro = np.concatenate(ro_all)
+    rm = oracle.sample(off, nbr, model, seed, 0, theta, nthreads=NT)[1]
+    assert int(ro[-1]) == rm.size
+    return ro, rm
+
+
+def test_C2_sets_exhaustive_coverage_and_imm(eim, ctx, graphs, monkeypatch):
+    # every RRR set of the IMM's R (ids [0, theta) = [0, 101294)), the
+    # per-vertex coverage counts C and the full IMM (the bench workload)
     c = inputs.CONFIGS["C2"]
     off, nbr = graphs("C2")
+    n = off.size - 1
     g = eim.eim_load_graph_csr(ctx, off, nbr)
     try:
-        _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 0, 3000)
-        assert eim.eim_get_stats(ctx)["spilled_samples"] > 0  # the heavy samples take the queue path
+        st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
+        assert st["theta"] == 101294
+        C_gpu = eim.eim_get_coverage(ctx, n)
+        ro, rm = _exhaustive(eim, ctx, g, off, nbr, "IC", 1, st["theta"])
+        assert np.array_equal(C_gpu, oracle.coverage(n, ro, rm))
+        assert int(C_gpu.sum()) == st["arena_elems"]
         with monkeypatch.context() as mp:
             mp.setenv("EIM_SPILL_QUADS", "1")
             mp.setenv("EIM_TASK_QUADS", "1")
@@ -219,19 +248,103 @@ def test_C2_sampled_sets_and_imm(eim, ctx, graphs, monkeypatch):
             mp.setenv("EIM_RING_W", "32")
             _sets_equal(eim, ctx, g, off, nbr, "IC", 1, 5555, 1000)
             assert eim.eim_get_stats(ctx)["spilled_samples"] > 0
-        st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
-        assert st["theta"] > 50000
     finally:
         eim.eim_graph_free(g)
 
 
-def test_C3_sampled_sets_and_imm(eim, ctx, graphs):
+def test_C3_sets_exhaustive_coverage_and_imm(eim, ctx, graphs):
     c = inputs.CONFIGS["C3"]
     off, nbr = graphs("C3")
+    n = off.size - 1
     g = eim.eim_load_graph_csr(ctx, off, nbr)
     try:
-        _sets_equal(eim, ctx, g, off, nbr, "LT", 1, 0, 20000)
-        _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
+        st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
+        assert st["theta"] == 58277
+        C_gpu = eim.eim_get_coverage(ctx, n)
+        ro, rm = _exhaustive(eim, ctx, g, off, nbr, "LT", 1, st["theta"])
+        assert np.array_equal(C_gpu, oracle.coverage(n, ro, rm))
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_C4_sets_and_imm(eim, ctx, graphs):
+    # Twitter-shaped (1.47e9 edges, max in-degree ~4e5): the full IMM against
+    # one full oracle IMM, the largest sets of R and a random id sample set by
+    # set, and C over a 20,000-id prefix (the IMM's full C needs every set).
+    c = inputs.CONFIGS["C4"]
+    off, nbr = graphs("C4")
+    n = off.size - 1
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "IC", 1)
+        go, gm = eim.eim_sample_rrr(ctx, g, "IC", 1, 0, 20000)
+        ro, rm, _ = oracle.sample(off, nbr, "IC", 1, 0, 20000, nthreads=NT)
+        assert np.array_equal(go, ro) and np.array_equal(gm, rm)
+        sizes = np.diff(ro)
+        big = np.argsort(-sizes.astype(np.int64), kind="stable")[:200]
+        rng = np.random.default_rng(4)
+        for s in sorted(set(big.tolist()) | set(rng.integers(20000, st["theta"], size=300).tolist())):
+            _sets_equal(eim, ctx, g, off, nbr, "IC", 1, int(s), 1)
+        s, gains = eim.eim_select_seeds(ctx, n, ro, rm, c["k"])
+        rs, rg, _ = oracle.greedy(n, ro, rm, c["k"])
+        assert np.array_equal(s, rs) and np.array_equal(gains, rg)
+        _coverage_equal(eim, ctx, n, ro, rm)
+    finally:
+        eim.eim_graph_free(g)
+
+
+# The martingale loop's stop test, LB and theta against their closed forms
+# (tests/test_oracle_imm.py: one vertex in every RRR set => cov_i = |R|),
+# evaluated in mpmath -- independent of the oracle.
+@pytest.mark.parametrize("shape", ["path", "star", "cycle"])
+def test_imm_stop_test_closed_form_gpu(eim, ctx, shape):
+    from test_oracle_imm import ALL_COVERED_CASES, ALL_COVERED_GRAPHS, closed_form_all_covered
+    for n, k, eps, ell in ALL_COVERED_CASES:
+        off, nbr = ALL_COVERED_GRAPHS[shape](n)
+        want = closed_form_all_covered(n, k, eps, ell)
+        g = eim.eim_load_graph_csr(ctx, off, nbr)
+        try:
+            for model in ("IC", "LT"):
+                seeds, theta, spread, st = eim.eim_imm_run(ctx, g, k, eps, ell, model, 11)
+                assert st["theta_i"] == want["theta_i"] and st["cov_i"] == want["theta_i"], (n, k, eps)
+                if want["lb"] is None:
+                    assert st["lb"] == 1.0
+                else:
+                    assert abs(st["lb"] - float(want["lb"])) <= 1e-12 * float(want["lb"])
+                assert theta == want["theta"] and st["cov"] == theta and spread == float(n)
+                assert seeds.tolist() == list(range(k))
+                C = eim.eim_get_coverage(ctx, n)
+                if shape == "cycle":
+                    assert np.array_equal(C, np.full(n, theta))
+                else:
+                    assert C[0] == theta
+        finally:
+            eim.eim_graph_free(g)
+
+
+def test_coverage_counts_C1_and_select(eim, ctx, graphs):
+    off, nbr = graphs("C1")
+    n = off.size - 1
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        for model in ("IC", "LT"):
+            for seed in (1, 2):
+                _, theta, _, _ = eim.eim_imm_run(ctx, g, 5, 0.5, 1.0, model, seed)
+                ro, rm, _ = oracle.sample(off, nbr, model, seed, 0, theta, nthreads=NT)
+                _coverage_equal(eim, ctx, n, ro, rm)
+            _, theta, _, _ = eim.eim_imm_run(ctx, g, 5, 0.5, 1.0, model, 3, flags=oracle.FRESH_FINAL)
+            ro, rm, _ = oracle.sample(off, nbr, model, 3, oracle.FRESH_BASE, theta, nthreads=NT)
+            _coverage_equal(eim, ctx, n, ro, rm)
+        eim.eim_sample_rrr(ctx, g, "IC", 1, 0, 10)
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_get_coverage(ctx, n)
+        assert ei.value.status == eim.EIM_E_STATE
+        ro, rm, _ = oracle.sample(off, nbr, "IC", 3, 0, 3000, nthreads=NT)
+        eim.eim_select_seeds(ctx, n, ro, rm, 7)
+        _coverage_equal(eim, ctx, n, ro, rm)
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_get_coverage(ctx, n + 1)
+        assert ei.value.status == eim.EIM_E_INVAL
     finally:
         eim.eim_graph_free(g)
 
