@@ -111,6 +111,22 @@ typedef struct {
 eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint64_t stream,
                       eim_ctx** out);
 eim_status eim_nccl_get_id(void* out /* EIM_NCCL_ID_BYTES */);
+/* eim_create_group: `world` contexts in ONE process, out[r] = rank r on CUDA
+ * device devices[r] (caller-allocated array of `world` pointers).  Devices
+ * may repeat: several ranks may share one GPU ("virtual ranks").  The ranks
+ * share an in-process communicator (host rendezvous + stream-ordered device
+ * copies) in place of NCCL and run exactly the multi-rank code of a
+ * one-process-per-GPU context: each rank samples a contiguous share of every
+ * round's sample ids, the shares are exchanged in rank (= sample-id) order,
+ * and every rank's result equals the 1-GPU run.  Collective calls
+ * (eim_imm_run, eim_imm_run_ex) must be made on all ranks concurrently, one
+ * host thread per rank; the other calls are local to their context.  If one
+ * rank's collective call fails, the others fail with EIM_E_NCCL instead of
+ * waiting, and the group is unusable afterwards (every later collective
+ * call fails).  Each context is released with eim_destroy.
+ * Errors: EIM_E_INVAL (NULL arguments, world < 1, a device < 0 or out of
+ * range), EIM_E_CUDA, EIM_E_NOMEM; on failure no context is left. */
+eim_status eim_create_group(const int* devices, int world, eim_ctx** out);
 void eim_destroy(eim_ctx* ctx);
 /* Message for the last failed call on ctx (or for the last failed
  * eim_create / host-only call when ctx is NULL).  Valid until the next call. */
@@ -177,10 +193,14 @@ eim_status eim_graph_bytes(const eim_graph* g, uint64_t* bytes);
  *   k in [1, n]; eps in (0, 1); ell > 0 (IMM failure exponent, default 1).
  *   seeds_out[k]: seed vertices in pick order.  theta_out: final |R|.
  *   spread_out: n * cov / |R| (RIS estimate).  stats_out nullable.
- * Multi-GPU contexts: every rank calls with identical arguments; each rank
- * samples a contiguous share of every round's new ids, the shares are
- * all-gathered over NCCL and the greedy runs replicated, so every rank
- * returns the same result, identical to a single-GPU run.
+ * Multi-rank contexts (NCCL or eim_create_group): every rank calls with
+ * identical arguments; each rank samples a contiguous share of every
+ * round's new ids, the shares are exchanged (all-gather of counts, one
+ * broadcast per share) and the greedy runs replicated, so every rank
+ * returns the same result, identical to a single-GPU run (also with
+ * EIM_F_SOURCE_ELIM: the first theta non-empty sets in sample-id order,
+ * wherever the cut falls).  stats_out->edges_examined, spilled_samples,
+ * sample_launches and the ms_* fields are this rank's.
  * Errors: EIM_E_INVAL, EIM_E_STATE (graph from another ctx / freed),
  * EIM_E_NOMEM, EIM_E_CUDA, EIM_E_NCCL.
  */
@@ -191,9 +211,8 @@ eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps,
 /* eim_imm_run_ex: eim_imm_run with run flags (EIM_F_SOURCE_ELIM |
  * EIM_F_FRESH_FINAL; 0 = eim_imm_run).  stats_out->ids_sampled counts the
  * sample ids drawn.  Errors: those of eim_imm_run, and EIM_E_INVAL for an
- * unknown flag, EIM_F_SOURCE_ELIM on a multi-GPU context, or
- * EIM_F_SOURCE_ELIM on a graph with no edge u -> v, u != v (every set would
- * be empty).
+ * unknown flag, or EIM_F_SOURCE_ELIM on a graph with no edge u -> v,
+ * u != v (every set would be empty).
  */
 eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell,
                           eim_model model, uint64_t seed, uint32_t flags, uint32_t* seeds_out,

@@ -29,7 +29,7 @@ STATUS_NAMES = {0: "EIM_OK", -1: "EIM_E_INVAL", -2: "EIM_E_NOMEM", -3: "EIM_E_CU
                 -5: "EIM_E_CAPACITY", -6: "EIM_E_STATE"}
 
 # Every symbol include/eim.h declares (checked by tests/test_abi.py).
-EXPORTS = ["eim_create", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "eim_version",
+EXPORTS = ["eim_create", "eim_create_group", "eim_nccl_get_id", "eim_destroy", "eim_last_error", "eim_version",
            "eim_load_graph_csr", "eim_load_graph_csr_ex", "eim_load_graph_csr_weighted", "eim_graph_bytes",
            "eim_graph_free", "eim_imm_run", "eim_imm_run_ex", "eim_sample_rrr",
            "eim_sample_rrr_ex", "eim_select_seeds",
@@ -94,6 +94,7 @@ def lib():
     sig = {
         "eim_create": (_I, [_I, _I, _I, _P, _U64, ctypes.POINTER(_P)]),
         "eim_nccl_get_id": (_I, [_P]),
+        "eim_create_group": (_I, [_P, _I, _P]),
         "eim_destroy": (None, [_P]),
         "eim_last_error": (ctypes.c_char_p, [_P]),
         "eim_version": (ctypes.c_char_p, []),
@@ -147,6 +148,15 @@ def eim_create(device=0, rank=0, world=1, nccl_id: bytes | None = None, stream: 
     idbuf = ctypes.create_string_buffer(nccl_id, NCCL_ID_BYTES) if nccl_id is not None else None
     _check(lib().eim_create(device, rank, world, idbuf, stream, ctypes.byref(out)))
     return out.value
+
+
+def eim_create_group(devices):
+    """In-process ranks (one context per entry of devices; devices may repeat).
+    Returns the list of contexts, rank order."""
+    devs = np.ascontiguousarray(list(devices), dtype=np.int32)
+    out = (_P * len(devs))()
+    _check(lib().eim_create_group(devs.ctypes.data, len(devs), out))
+    return [out[r] for r in range(len(devs))]
 
 
 def eim_destroy(ctx):

@@ -114,6 +114,58 @@ eim_status eim_nccl_get_id(void* out) {
   });
 }
 
+}  // extern "C"
+
+namespace {
+
+// A context on `device`; the communicator is made by make_comm (world > 1).
+template <class MakeComm>
+eim_ctx* new_ctx(int device, int rank, int world, uint64_t stream, MakeComm&& make_comm) {
+  int ndev = 0;
+  EIM_CUDA(cudaGetDeviceCount(&ndev));
+  if (device >= ndev) fail(EIM_E_INVAL, "device index out of range");
+  EIM_CUDA(cudaSetDevice(device));
+  eim_ctx* c = new eim_ctx();
+  c->magic = CTX_MAGIC;
+  c->device = device;
+  c->rank = rank;
+  c->world = world;
+  c->comm = nullptr;
+  c->kernel_launches = 0;
+  c->own_stream = stream == 0;
+  try {
+    if (c->own_stream) EIM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+    else c->stream = reinterpret_cast<cudaStream_t>(stream);
+    EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[0], cudaStreamNonBlocking));
+    EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
+    EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
+    EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
+    // keep freed stream-ordered memory in the device's pool: reloading a
+    // graph or regrowing a buffer reuses it instead of cudaMalloc/cudaFree
+    cudaMemPool_t pool;
+    EIM_CUDA(cudaDeviceGetDefaultMemPool(&pool, device));
+    uint64_t keep_all = UINT64_MAX;
+    EIM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep_all));
+    EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
+    EIM_CUDA(cudaEventCreate(&c->ev0));
+    EIM_CUDA(cudaEventCreate(&c->ev1));
+    c->scratch.reserve(1 << 20, false, c->stream);
+    if (world > 1) c->comm = make_comm();
+  } catch (...) {
+    free_ctx_buffers(c);
+    if (c->h_pinned) cudaFreeHost(c->h_pinned);
+    if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+    c->magic = 0;
+    delete c;
+    throw;
+  }
+  return c;
+}
+
+}  // namespace
+
+extern "C" {
+
 eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint64_t stream, eim_ctx** out) {
   return guarded(nullptr, [&] {
     if (!out) fail(EIM_E_INVAL, "out is NULL");
@@ -121,45 +173,33 @@ eim_status eim_create(int device, int rank, int world, const void* nccl_id, uint
     if (device < 0) fail(EIM_E_INVAL, "device < 0");
     if (world < 1 || rank < 0 || rank >= world) fail(EIM_E_INVAL, "rank/world out of range");
     if (world > 1 && !nccl_id) fail(EIM_E_INVAL, "world > 1 needs an NCCL unique id");
-    int ndev = 0;
-    EIM_CUDA(cudaGetDeviceCount(&ndev));
-    if (device >= ndev) fail(EIM_E_INVAL, "device index out of range");
-    EIM_CUDA(cudaSetDevice(device));
-    eim_ctx* c = new eim_ctx();
-    c->magic = CTX_MAGIC;
-    c->device = device;
-    c->rank = rank;
-    c->world = world;
-    c->comm = nullptr;
-    c->kernel_launches = 0;
-    c->own_stream = stream == 0;
+    *out = new_ctx(device, rank, world, stream, [&] { return comm_create(rank, world, nccl_id); });
+  });
+}
+
+eim_status eim_create_group(const int* devices, int world, eim_ctx** out) {
+  return guarded(nullptr, [&] {
+    if (!out || !devices) fail(EIM_E_INVAL, "NULL argument");
+    if (world < 1) fail(EIM_E_INVAL, "world < 1");
+    for (int r = 0; r < world; ++r) {
+      out[r] = nullptr;
+      if (devices[r] < 0) fail(EIM_E_INVAL, "device < 0");
+    }
+    LocalGroup* grp = world > 1 ? local_group_new(world) : nullptr;
+    int made = 0;
     try {
-      if (c->own_stream) EIM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
-      else c->stream = reinterpret_cast<cudaStream_t>(stream);
-      EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[0], cudaStreamNonBlocking));
-      EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
-      EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
-      EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
-      // keep freed stream-ordered memory in the device's pool: reloading a
-      // graph or regrowing a buffer reuses it instead of cudaMalloc/cudaFree
-      cudaMemPool_t pool;
-      EIM_CUDA(cudaDeviceGetDefaultMemPool(&pool, device));
-      uint64_t keep_all = UINT64_MAX;
-      EIM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep_all));
-      EIM_CUDA(cudaMallocHost(&c->h_pinned, 4096));
-      EIM_CUDA(cudaEventCreate(&c->ev0));
-      EIM_CUDA(cudaEventCreate(&c->ev1));
-      c->scratch.reserve(1 << 20, false, c->stream);
-      if (world > 1) c->comm = comm_create(rank, world, nccl_id);
+      for (int r = 0; r < world; ++r) {
+        out[r] = new_ctx(devices[r], r, world, 0, [&] { return comm_create_local(grp, r); });
+        made++;
+      }
     } catch (...) {
-      free_ctx_buffers(c);
-      if (c->h_pinned) cudaFreeHost(c->h_pinned);
-      if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
-      c->magic = 0;
-      delete c;
+      for (int r = 0; r < made; ++r) {
+        eim_destroy(out[r]);
+        out[r] = nullptr;
+      }
+      if (grp && made == 0) delete_local_group(grp);
       throw;
     }
-    *out = c;
   });
 }
 
@@ -286,16 +326,23 @@ eim_status eim_imm_run_ex(eim_ctx* ctx, const eim_graph* g, uint32_t k, double e
                           double* spread_out, eim_stats* stats_out) {
   if (!ctx_ok(ctx)) return EIM_E_STATE;
   return guarded(ctx, [&] {
-    check_graph(ctx, g);
-    if (flags & ~(uint32_t)(EIM_F_SOURCE_ELIM | EIM_F_FRESH_FINAL)) fail(EIM_E_INVAL, "unknown flag");
-    if (!seeds_out) fail(EIM_E_INVAL, "seeds_out is NULL");
-    if (k == 0 || k > g->view.n) fail(EIM_E_INVAL, "k must be in [1, n]");
-    if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
-    if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
-    if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
-    if (model == EIM_LT && !g->lt_ok) fail(EIM_E_INVAL, "LT: a row's edge weights sum to more than 1");
-    ctx->cov_n = 0;
-    imm_run(ctx, g, k, eps, ell, model, seed, flags, seeds_out, theta_out, spread_out, &ctx->last_stats);
+    try {
+      check_graph(ctx, g);
+      if (flags & ~(uint32_t)(EIM_F_SOURCE_ELIM | EIM_F_FRESH_FINAL)) fail(EIM_E_INVAL, "unknown flag");
+      if (!seeds_out) fail(EIM_E_INVAL, "seeds_out is NULL");
+      if (k == 0 || k > g->view.n) fail(EIM_E_INVAL, "k must be in [1, n]");
+      if (!(eps > 0.0 && eps < 1.0)) fail(EIM_E_INVAL, "eps must be in (0, 1)");
+      if (!(ell > 0.0)) fail(EIM_E_INVAL, "ell must be > 0");
+      if (model != EIM_IC && model != EIM_LT) fail(EIM_E_INVAL, "unknown model");
+      if (model == EIM_LT && !g->lt_ok) fail(EIM_E_INVAL, "LT: a row's edge weights sum to more than 1");
+      ctx->cov_n = 0;
+      imm_run(ctx, g, k, eps, ell, model, seed, flags, seeds_out, theta_out, spread_out, &ctx->last_stats);
+    } catch (...) {
+      // a collective call: release the peers of a local group (they would
+      // wait for this rank forever); the group cannot be used afterwards
+      if (ctx->comm) ctx->comm->abort();
+      throw;
+    }
     ctx->cov_n = g->view.n;
     if (stats_out) *stats_out = ctx->last_stats;
   });

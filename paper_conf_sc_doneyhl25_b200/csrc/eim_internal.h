@@ -82,7 +82,23 @@ struct SampleCtl {
   unsigned long long pad4[8];
 };
 
-struct Comm;  // NCCL communicator wrapper (comm.cpp)
+// Communicator of a multi-rank context (comm.cpp): NCCL across processes,
+// or an in-process group of ranks (eim_create_group).  Collectives are
+// stream-ordered on `st`; every rank calls them in the same order.
+struct Comm {
+  int rank = 0, world = 1;
+  virtual ~Comm();
+  // d_recv[q] = rank q's *d_send (one u64 per rank)
+  virtual void allgather_u64(const uint64_t* d_send, uint64_t* d_recv, cudaStream_t st) = 0;
+  // every rank's d_buf[0, bytes) = root's
+  virtual void broadcast(void* d_buf, size_t bytes, int root, cudaStream_t st) = 0;
+  virtual void group_start() {}
+  virtual void group_end() {}
+  // this rank failed: release the peers waiting in a collective (local groups)
+  virtual void abort() {}
+  virtual const char* kind() const = 0;
+};
+struct LocalGroup;
 
 // One sampler launch over sample ids [first, first+count): its membership
 // table and per-sample scratch.  Two of them let the IMM driver sample the
@@ -91,6 +107,15 @@ struct Comm;  // NCCL communicator wrapper (comm.cpp)
 // its set; with RF_DROP_EMPTY the sets left empty are discarded and only
 // the first `use` non-empty sets (in sample-id order) are kept.
 enum : uint32_t { RF_DROP_ROOT = 1u, RF_DROP_EMPTY = 2u };
+
+struct SampleResult {
+  uint64_t edges = 0;
+  uint64_t spilled = 0;   // samples finished in the shared frontier queue
+  uint32_t launches = 0;
+  double kernel_ms = 0;
+  uint64_t kept = 0;      // sets appended to the arena
+  uint64_t consumed = 0;  // sample ids used (> kept when empty sets are dropped)
+};
 
 struct Round {
   DevBuf table, sizes, edges, fill, excl, ctl;  // ctl: SampleCtl + cancel/pause flags
@@ -109,6 +134,9 @@ struct Round {
   bool waited = false;  // the launch has finished (round_finalize with keep appends the rest later)
   bool hist = true;
   uint32_t rflags = 0;
+  SampleResult pend;          // launch statistics not yet reported by round_finalize
+  bool elim_ready = false;    // RF_DROP_EMPTY: roots dropped from the sizes, kidx scanned (round_elim_kept)
+  uint64_t kept_total = 0;    // RF_DROP_EMPTY: non-empty sets of the launch
 };
 
 }  // namespace eim
@@ -181,14 +209,6 @@ void graph_attach_weights(eim_ctx* ctx, eim_graph* g, const uint32_t* h_x);
 bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g);
 
 // ---- sample.cu
-struct SampleResult {
-  uint64_t edges = 0;
-  uint64_t spilled = 0;   // samples finished in the shared frontier queue
-  uint32_t launches = 0;
-  double kernel_ms = 0;
-  uint64_t kept = 0;      // sets appended to the arena
-  uint64_t consumed = 0;  // sample ids used (> kept when empty sets are dropped)
-};
 // Samples ids [first, first+count) into ctx->arena; set index = id - set_base.
 // Histogram into C when hist is true.  (= round_launch + round_finalize)
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
@@ -204,8 +224,14 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 // is the number of non-empty sets wanted (res.kept <= use, res.consumed ids).
 // from/keep: append only s_local in [from, use) and keep the round for a
 // later append of the rest (plain rounds; the IMM driver's lookahead).
+// consume_all (RF_DROP_EMPTY, use = every non-empty set of the launch): all
+// ids of the launch count as consumed (a multi-rank round whose cut lies on
+// a later rank).
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from = 0,
-                            bool keep = false);
+                            bool keep = false, bool consume_all = false);
+// RF_DROP_EMPTY rounds: wait, drop the roots and count the non-empty sets
+// of the whole launch (idempotent; round_finalize then keeps the first `use`).
+uint64_t round_elim_kept(eim_ctx* ctx, const eim_graph* g, Round& rd);
 // Stop a launched speculative round and wait for it.
 void round_cancel(eim_ctx* ctx, Round& rd);
 // Let a launched round take no new sample ids (its running samples finish);
@@ -246,13 +272,12 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
              eim_stats* st);
 
 // ---- comm.cpp
-Comm* comm_create(int rank, int world, const void* id);
+Comm* comm_create(int rank, int world, const void* id);  // NCCL
+LocalGroup* local_group_new(int world);
+void delete_local_group(LocalGroup* grp);                // only if no comm holds it
+Comm* comm_create_local(LocalGroup* grp, int rank);      // takes a reference on grp
 void comm_destroy(Comm* c);
 void comm_get_id(void* out);
-void comm_allgather_u64(Comm* c, const uint64_t* d_send, uint64_t* d_recv, cudaStream_t st);
-void comm_broadcast(Comm* c, void* d_buf, size_t bytes, int root, cudaStream_t st);
-void comm_group_start();
-void comm_group_end();
 
 inline uint32_t grid_for(eim_ctx* ctx, uint64_t work, uint32_t per_block, uint32_t blocks_per_sm = 8) {
   uint64_t b = (work + per_block - 1) / per_block;

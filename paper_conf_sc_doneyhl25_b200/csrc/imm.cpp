@@ -43,91 +43,108 @@ double ms_since(clk::time_point t0) {
 }
 
 struct Exchange {
-  DevBuf counts, offs_recv, mem_recv, len_send;
+  DevBuf counts, offs_recv, mem_recv;
 };
 
-// Sets [R, R_new) (sample ids id_base + set index) across ranks; afterwards
-// every rank holds all of them.
-void sample_round(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, uint64_t id_base, uint64_t R,
-                  uint64_t R_new, eim_stats* st, Exchange& ex) {
+// After this every rank holds the sets [a, b): rank q contributes its part
+// parts[q] (set indices; the parts are contiguous, in rank order = sample-id
+// order, and cover [a, b)), which it has already appended to its own arena.
+// Each rank compacts its part, the member counts are all-gathered and every
+// part is broadcast from its owner and appended by the others; then every
+// rank adds the histogram of the whole range to C (the rounds of a
+// multi-rank context are launched without it).
+void exchange_sets(eim_ctx* ctx, uint64_t a, uint64_t b, const std::vector<std::pair<uint64_t, uint64_t>>& parts,
+                   Exchange& ex, eim_stats* st) {
   const auto t0 = clk::now();
   cudaStream_t s = ctx->stream;
-  uint64_t lo, hi;
-  eim_shard_range(R, R_new - R, ctx->rank, ctx->world, &lo, &hi);
-  SampleResult r = sample_range(ctx, g, model, seed, id_base + lo, hi - lo, id_base, false);
-  st->edges_examined += r.edges;
-  st->spilled_samples += r.spilled;
-  st->sample_launches += r.launches;
-  st->ms_sample_kernel += r.kernel_ms;
-  const auto tc = clk::now();
-  ensure_sets(ctx, R_new);
-  // own share, compacted in sample-id order (offsets relative to the share)
+  Comm* comm = ctx->comm;
+  const int W = ctx->world, me = ctx->rank;
+  for (int q = 0; q < W; ++q)
+    if (parts[q].second < parts[q].first || parts[q].first != (q ? parts[q - 1].second : a) ||
+        (q == W - 1 && parts[q].second != b))
+      fail(EIM_E_STATE, "exchange_sets: parts are not a rank-ordered partition of the range");
+  ensure_sets(ctx, b);
   uint64_t* d_off = nullptr;
   uint32_t* d_mem = nullptr;
-  const uint64_t my_total = compact_range(ctx, lo, hi - lo, &d_off, &d_mem);
-  const int W = ctx->world;
+  const uint64_t my_total = compact_range(ctx, parts[me].first, parts[me].second - parts[me].first, &d_off, &d_mem);
   ex.counts.reserve(2 * W * sizeof(uint64_t), false, s);
   uint64_t* d_counts = ex.counts.as<uint64_t>();
   EIM_CUDA(cudaMemcpyAsync(d_counts, &my_total, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
-  comm_allgather_u64(ctx->comm, d_counts, d_counts + W, s);
+  comm->allgather_u64(d_counts, d_counts + W, s);
   std::vector<uint64_t> totals(W);
   EIM_CUDA(cudaMemcpyAsync(totals.data(), d_counts + W, W * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   EIM_CUDA(cudaStreamSynchronize(s));
   uint64_t max_total = 1, max_sets = 1;
   for (int q = 0; q < W; ++q) {
-    uint64_t a, b;
-    eim_shard_range(R, R_new - R, q, W, &a, &b);
     max_total = std::max(max_total, totals[q]);
-    max_sets = std::max(max_sets, b - a + 1);
+    max_sets = std::max(max_sets, parts[q].second - parts[q].first + 1);
   }
   ex.offs_recv.reserve(max_sets * sizeof(uint64_t), false, s);
   ex.mem_recv.reserve(max_total * sizeof(uint32_t), false, s);
   for (int q = 0; q < W; ++q) {
-    uint64_t a, b;
-    eim_shard_range(R, R_new - R, q, W, &a, &b);
-    if (b == a) continue;
-    uint64_t* offs = (q == ctx->rank) ? d_off : ex.offs_recv.as<uint64_t>();
-    uint32_t* mem = (q == ctx->rank) ? d_mem : ex.mem_recv.as<uint32_t>();
-    comm_group_start();
-    comm_broadcast(ctx->comm, offs, (b - a + 1) * sizeof(uint64_t), q, s);
-    if (totals[q]) comm_broadcast(ctx->comm, mem, totals[q] * sizeof(uint32_t), q, s);
-    comm_group_end();
-    if (q != ctx->rank) append_sets(ctx, a, b - a, offs, mem, totals[q]);
+    const uint64_t pa = parts[q].first, pb = parts[q].second;
+    if (pb == pa) continue;
+    uint64_t* offs = (q == me) ? d_off : ex.offs_recv.as<uint64_t>();
+    uint32_t* mem = (q == me) ? d_mem : ex.mem_recv.as<uint32_t>();
+    comm->group_start();
+    comm->broadcast(offs, (pb - pa + 1) * sizeof(uint64_t), q, s);
+    if (totals[q]) comm->broadcast(mem, totals[q] * sizeof(uint32_t), q, s);
+    comm->group_end();
+    if (q != me) append_sets(ctx, pa, pb - pa, offs, mem, totals[q]);
   }
-  hist_sets(ctx, R, R_new);
+  hist_sets(ctx, a, b);
   EIM_CUDA(cudaStreamSynchronize(s));
-  st->ms_comm += ms_since(tc);
-  st->ms_sample += ms_since(t0);
+  st->ms_comm += ms_since(t0);
 }
 
-// Supplies the sets of sample ids [|R|, to) to the arena.  On one GPU the
-// next round's ids [to, next_to) are launched SPECULATIVELY on a second
-// stream right behind the current round's launch: its blocks take the SMs
-// that the current round's tail (its last, longest reverse-BFS chains)
-// leaves idle.  While the greedy of the current round runs, the speculative
-// round is paused (it takes no new ids, so the greedy has the GPU); it is
-// resumed when its ids are needed, or cancelled when they are not.  Sample
-// ids are fixed labels, so a speculative set is exactly the set the next
-// round needs and results are unchanged.
+// all-gather of one host u64 per rank
+std::vector<uint64_t> allgather_host(eim_ctx* ctx, Exchange& ex, uint64_t v) {
+  const int W = ctx->world;
+  std::vector<uint64_t> out(W, v);
+  if (W == 1) return out;
+  cudaStream_t s = ctx->stream;
+  ex.counts.reserve(2 * W * sizeof(uint64_t), false, s);
+  uint64_t* d = ex.counts.as<uint64_t>();
+  EIM_CUDA(cudaMemcpyAsync(d, &v, sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+  ctx->comm->allgather_u64(d, d + W, s);
+  EIM_CUDA(cudaMemcpyAsync(out.data(), d + W, W * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  EIM_CUDA(cudaStreamSynchronize(s));
+  return out;
+}
+
+// Supplies the sets of sample ids [|R|, to) to the arena.
+//
+// Every rank of a W-rank context (W = 1 on one GPU) launches its contiguous
+// share (eim_shard_range) of a launch range [first, end) and appends its
+// part of each requested range [|R|, to); with W > 1 the parts are then
+// exchanged (exchange_sets), so every rank holds all sets in sample-id order.
+//
+// Lookahead (default on; EIM_NO_LOOKAHEAD=1 turns it off): when the next
+// estimation round adds no more ids than this one, one launch samples both
+// and the next round's sets are appended from the same round table without a
+// launch -- one round tail (the heavy samples' critical paths; for LT the
+// longest walk) instead of two.  Sample ids are fixed labels, so the sets
+// are the same; if the estimation loop stops first the extra sets are
+// discarded.
+//
+// Speculation (opt-in EIM_SPECULATE=1, one GPU): the next round's ids are
+// launched on a second stream right behind the current round's launch and
+// paused while the greedy runs (measured on C2: the speculative round slows
+// the current round's critical chains as much as it fills their idle SMs).
 //
 // Source elimination (R22, elim = true): sets are the non-empty root-less
 // sets in sample-id order; a round launches enough ids for the sets still
-// needed (from the kept fraction so far), keeps the first of them and
-// continues from the id after the last kept one.
+// needed (from the kept fraction so far); every rank counts the non-empty
+// sets of its share, the counts are all-gathered, and the cut (the id of the
+// |R|-th kept set) falls in one rank's share: the ranks before it keep all
+// their sets and consume all their ids, the cut rank keeps a prefix, the
+// ranks after it keep and consume nothing.
 class RoundSampler {
  public:
   RoundSampler(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed, eim_stats* st, bool elim)
       : ctx_(ctx), g_(g), model_(model), seed_(seed), st_(st), elim_(elim) {
-    // opt-in (EIM_SPECULATE=1): measured on C2 the speculative round slows the
-    // current round's critical chains as much as it fills their idle SMs
     speculate_ = ctx->world == 1 && !elim && std::getenv("EIM_SPECULATE") != nullptr;
-    // Lookahead (default on, one GPU, plain runs): when the next round adds no
-    // more ids than this one, one launch samples both and the next round's
-    // sets are appended from the same round table without a launch -- one
-    // round tail (the heavy samples' critical paths) instead of two.  Sample
-    // ids are fixed labels, so the sets are the same; if the estimation loop
-    // stops first, the extra sets are discarded.  EIM_NO_LOOKAHEAD=1: off.
-    lookahead_ = ctx->world == 1 && !elim && !speculate_ && std::getenv("EIM_NO_LOOKAHEAD") == nullptr;
+    lookahead_ = !elim && !speculate_ && std::getenv("EIM_NO_LOOKAHEAD") == nullptr;
   }
 
   // Continue with an empty arena from sample id `id_base` (fresh final phase, R23).
@@ -142,54 +159,19 @@ class RoundSampler {
     ex_.mem_recv.release();
   }
 
-  // make sets [R, to) final; speculate [to, next_to)
+  // make sets [R, to) final; next_to: the next round's target (lookahead / speculation)
   void grow(uint64_t& R, uint64_t to, uint64_t next_to) {
     if (to <= R) return;
     const auto t0 = clk::now();
     if (elim_) {
       grow_elim(R, to);
-      st_->ms_sample += ms_since(t0);
-      return;
-    }
-    st_->ids_sampled += to - R;
-    if (ctx_->world > 1) {
-      sample_round(ctx_, g_, model_, seed_, id_base_, R, to, st_, ex_);
-      R = to;
-      return;
-    }
-    if (lookahead_) {
-      grow_lookahead(R, to, next_to);
-      st_->ms_sample += ms_since(t0);
-      return;
-    }
-    Round* cur = nullptr;
-    if (spec_ && spec_->first == id_base_ + R) {
-      cur = spec_;
-      spec_ = nullptr;
-      round_resume(ctx_, g_, *cur, stream_of(*cur));
+    } else if (speculate_) {
+      st_->ids_sampled += to - R;
+      grow_speculate(R, to, next_to);
     } else {
-      cancel();
-      cur = &ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, *cur, stream_of(*cur), false);
+      st_->ids_sampled += to - R;
+      grow_shared(R, to, next_to);
     }
-    const uint64_t cur_end = R + cur->count;
-    if (speculate_ && next_to > cur_end) {
-      Round& nx = (cur == &ctx_->rounds[0]) ? ctx_->rounds[1] : ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, id_base_ + cur_end, next_to - cur_end, id_base_, true, nx, stream_of(nx),
-                   true);
-      spec_ = &nx;
-    }
-    const uint64_t use = std::min<uint64_t>(cur->count, to - R);
-    account(round_finalize(ctx_, g_, *cur, use));
-    R += use;
-    if (to > R) {  // the speculative range was shorter than needed: sample the rest now
-      cancel();
-      Round& rd = ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, rd, stream_of(rd), false);
-      account(round_finalize(ctx_, g_, rd, to - R));
-      R = to;
-    }
-    if (spec_ && !std::getenv("EIM_SPEC_NOPAUSE")) round_pause(ctx_, *spec_);
     st_->ms_sample += ms_since(t0);
   }
 
@@ -209,34 +191,53 @@ class RoundSampler {
     st_->sample_launches += r.launches;
     st_->ms_sample_kernel += r.kernel_ms;
   }
-  // The held launch covers ids id_base_ + [held_first_, held_end_); sets
-  // [held_first_, held_done_) are appended.
-  void grow_lookahead(uint64_t& R, uint64_t to, uint64_t next_to) {
-    Round& rd = ctx_->rounds[0];
+  int W() const { return ctx_->world; }
+
+  // ---- plain runs, any number of ranks.  The held launch covers set
+  // indices [launch_first_, launch_end_) (this rank: [my_lo_, my_hi_));
+  // sets [launch_first_, held_done_) are appended on every rank.
+  void grow_shared(uint64_t& R, uint64_t to, uint64_t next_to) {
     if (held_) {
       if (held_done_ == R) {
-        const uint64_t upto = std::min(held_end_, to);
-        const bool keep = upto < held_end_;
-        account(round_finalize(ctx_, g_, rd, upto - held_first_, held_done_ - held_first_, keep));
-        R = held_done_ = upto;
-        if (!keep) held_ = false;
+        append_part(R, std::min(launch_end_, to));
+        R = held_done_;
       } else {
         drop_held();
       }
     }
     if (to <= R) return;
     drop_held();
-    const uint64_t end = (next_to > to && next_to - to <= to - R) ? next_to : to;
-    round_launch(ctx_, g_, model_, seed_, id_base_ + R, end - R, id_base_, true, rd, stream_of(rd), false);
-    const bool keep = end > to;
-    account(round_finalize(ctx_, g_, rd, to - R, 0, keep));
-    if (keep) {
-      held_ = true;
-      held_first_ = R;
-      held_done_ = to;
-      held_end_ = end;
-    }
+    const uint64_t end = (lookahead_ && next_to > to && next_to - to <= to - R) ? next_to : to;
+    launch_first_ = R;
+    launch_end_ = end;
+    eim_shard_range(R, end - R, ctx_->rank, W(), &my_lo_, &my_hi_);
+    Round& rd = ctx_->rounds[0];
+    if (my_hi_ > my_lo_)
+      round_launch(ctx_, g_, model_, seed_, id_base_ + my_lo_, my_hi_ - my_lo_, id_base_, W() == 1, rd, stream_of(rd),
+                   false);
+    held_ = true;
+    held_done_ = R;
+    append_part(R, to);
     R = to;
+  }
+
+  // Append the sets [a, b) of the held launch (a = held_done_) on every rank.
+  void append_part(uint64_t a, uint64_t b) {
+    Round& rd = ctx_->rounds[0];
+    auto clampr = [](uint64_t x, uint64_t lo, uint64_t hi) { return std::min(std::max(x, lo), hi); };
+    const uint64_t pa = clampr(a, my_lo_, my_hi_), pb = clampr(b, my_lo_, my_hi_);
+    if (my_hi_ > my_lo_ && rd.launched) account(round_finalize(ctx_, g_, rd, pb - my_lo_, pa - my_lo_, pb < my_hi_));
+    if (W() > 1) {
+      std::vector<std::pair<uint64_t, uint64_t>> parts(W());
+      for (int q = 0; q < W(); ++q) {
+        uint64_t lo, hi;
+        eim_shard_range(launch_first_, launch_end_ - launch_first_, q, W(), &lo, &hi);
+        parts[q] = {clampr(lo, a, b), clampr(hi, a, b)};  // [max(a, lo), min(b, hi)), empty parts at their place
+      }
+      exchange_sets(ctx_, a, b, parts, ex_, st_);
+    }
+    held_done_ = b;
+    if (b >= launch_end_) drop_held();
   }
 
   // Discard the rest of a held launch (the loop stopped or moved on).
@@ -248,24 +249,92 @@ class RoundSampler {
     held_ = false;
   }
 
+  // ---- one GPU, EIM_SPECULATE=1
+  void grow_speculate(uint64_t& R, uint64_t to, uint64_t next_to) {
+    Round* cur = nullptr;
+    if (spec_ && spec_->first == id_base_ + R) {
+      cur = spec_;
+      spec_ = nullptr;
+      round_resume(ctx_, g_, *cur, stream_of(*cur));
+    } else {
+      cancel();
+      cur = &ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, *cur, stream_of(*cur), false);
+    }
+    const uint64_t cur_end = R + cur->count;
+    if (next_to > cur_end) {
+      Round& nx = (cur == &ctx_->rounds[0]) ? ctx_->rounds[1] : ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, id_base_ + cur_end, next_to - cur_end, id_base_, true, nx, stream_of(nx),
+                   true);
+      spec_ = &nx;
+    }
+    const uint64_t use = std::min<uint64_t>(cur->count, to - R);
+    account(round_finalize(ctx_, g_, *cur, use));
+    R += use;
+    if (to > R) {  // the speculative range was shorter than needed: sample the rest now
+      cancel();
+      Round& rd = ctx_->rounds[0];
+      round_launch(ctx_, g_, model_, seed_, id_base_ + R, to - R, id_base_, true, rd, stream_of(rd), false);
+      account(round_finalize(ctx_, g_, rd, to - R));
+      R = to;
+    }
+    if (spec_ && !std::getenv("EIM_SPEC_NOPAUSE")) round_pause(ctx_, *spec_);
+  }
+
+  // ---- source elimination, any number of ranks
   void grow_elim(uint64_t& R, uint64_t to) {
     while (R < to) {
       const uint64_t need = to - R;
       // kept fraction so far (first launch: 1/4), 5% + 64 ids of slack
       const double q = consumed_ ? std::max(1e-6, (double)std::max<uint64_t>(kept_, 1) / (double)consumed_) : 0.25;
       const double want = std::ceil((double)need / q * 1.05) + 64.0;
-      const uint64_t count = (uint64_t)std::min(want, (double)(1ull << 29));
+      const uint64_t count = (uint64_t)std::min(want, (double)(1ull << 29) * W());
       if (next_id_ + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids exhausted (< 2^62)");
+      uint64_t lo, hi;
+      eim_shard_range(next_id_, count, ctx_->rank, W(), &lo, &hi);
       Round& rd = ctx_->rounds[0];
-      round_launch(ctx_, g_, model_, seed_, next_id_, count, next_id_ - R, true, rd, stream_of(rd), false,
-                   RF_DROP_ROOT | RF_DROP_EMPTY);
-      const SampleResult r = round_finalize(ctx_, g_, rd, need);
-      account(r);
-      R += r.kept;
-      next_id_ += r.consumed;
-      kept_ += r.kept;
-      consumed_ += r.consumed;
-      st_->ids_sampled += r.consumed;
+      if (hi > lo)
+        round_launch(ctx_, g_, model_, seed_, lo, hi - lo, lo, W() == 1, rd, stream_of(rd), false,
+                     RF_DROP_ROOT | RF_DROP_EMPTY);
+      const uint64_t kept_mine = (hi > lo) ? round_elim_kept(ctx_, g_, rd) : 0;
+      const std::vector<uint64_t> kept = allgather_host(ctx_, ex_, kept_mine);
+      // the cut: rank c holds the need-th kept set (none if too few were kept)
+      int c = -1;
+      uint64_t prefix = 0, my_base = 0, my_take = 0;
+      std::vector<std::pair<uint64_t, uint64_t>> parts(W());
+      for (int r = 0; r < W(); ++r) {
+        const uint64_t take = std::min(kept[r], need - std::min(need, prefix));
+        if (c < 0 && prefix + kept[r] >= need) c = r;
+        parts[r] = {R + std::min(prefix, need), R + std::min(prefix, need) + take};
+        if (r == ctx_->rank) {
+          my_base = R + std::min(prefix, need);
+          my_take = take;
+        }
+        prefix += kept[r];
+      }
+      const uint64_t taken = std::min(prefix, need);
+      const bool consume_all = c < 0 || ctx_->rank < c;
+      SampleResult r{};
+      if (hi > lo) {
+        rd.set_base = lo - my_base;  // this rank's kept set j goes to set index my_base + j
+        ensure_sets(ctx_, R + taken);
+        r = round_finalize(ctx_, g_, rd, my_take, 0, false, consume_all);
+        account(r);
+      }
+      // ids consumed by the whole round: everything up to the cut rank's cut
+      uint64_t gconsumed = count;
+      if (c >= 0) {
+        const std::vector<uint64_t> cons = allgather_host(ctx_, ex_, ctx_->rank == c ? r.consumed : 0);
+        uint64_t clo, chi;
+        eim_shard_range(next_id_, count, c, W(), &clo, &chi);
+        gconsumed = (clo - next_id_) + cons[c];
+      }
+      if (W() > 1) exchange_sets(ctx_, R, R + taken, parts, ex_, st_);
+      R += taken;
+      next_id_ += gconsumed;
+      kept_ += taken;
+      consumed_ += gconsumed;
+      st_->ids_sampled += gconsumed;
     }
   }
 
@@ -277,12 +346,12 @@ class RoundSampler {
   bool elim_;
   uint64_t id_base_ = 0;              // sample id of set index 0 (plain runs)
   uint64_t next_id_ = 0;              // next sample id (source elimination)
-  uint64_t kept_ = 0, consumed_ = 0;  // kept sets / ids used so far (source elimination)
+  uint64_t kept_ = 0, consumed_ = 0;  // kept sets / ids used so far (source elimination, all ranks)
   Exchange ex_;
   bool speculate_ = false;
   Round* spec_ = nullptr;
   bool lookahead_ = false, held_ = false;
-  uint64_t held_first_ = 0, held_done_ = 0, held_end_ = 0;
+  uint64_t launch_first_ = 0, launch_end_ = 0, held_done_ = 0, my_lo_ = 0, my_hi_ = 0;
 };
 
 }  // namespace
@@ -293,7 +362,6 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   const auto t_start = clk::now();
   const uint32_t n = g->view.n;
   const bool elim = (flags & EIM_F_SOURCE_ELIM) != 0, fresh = (flags & EIM_F_FRESH_FINAL) != 0;
-  if (elim && ctx->world > 1) fail(EIM_E_INVAL, "EIM_F_SOURCE_ELIM needs a single-GPU context");
   if (elim && !graph_has_proper_edge(ctx, g))
     fail(EIM_E_INVAL, "EIM_F_SOURCE_ELIM: the graph has no edge u->v with u != v (every set would be empty)");
   eim_imm_params_t p;

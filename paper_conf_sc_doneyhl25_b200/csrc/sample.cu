@@ -1329,6 +1329,7 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
   }
   rd.nlaunch = 0;
   rd.waited = false;
+  rd.elim_ready = false;
   round_kernel(ctx, g, rd, st, spare_sm_slot);
 }
 
@@ -1358,6 +1359,7 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   rd.first = first;
   rd.count = count;
   rd.set_base = set_base;
+  rd.pend = SampleResult{};
   rd.seed = seed;
   rd.model = model;
   rd.hist = hist;
@@ -1385,11 +1387,9 @@ void round_cancel(eim_ctx* ctx, Round& rd) {
   rd.qdirty = true;  // items may be left in the queue
 }
 
-SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from, bool keep) {
-  SampleResult res;
-  if (!rd.launched || rd.count == 0) return res;
-  if (use > rd.count || from > use) fail(EIM_E_STATE, "round_finalize beyond the launched range");
-  if (from > 0 && (rd.rflags & RF_DROP_ROOT)) fail(EIM_E_STATE, "partial appends of an eliminating round");
+// Wait for rd's launches (resuming a paused round), redo an overflowed round
+// with a larger table; accumulates the launch statistics in rd.pend.
+static void round_wait(eim_ctx* ctx, const eim_graph* g, Round& rd) {
   cudaStream_t st = ctx->stream;
   SampleCtl* ctl = rd.ctl.as<SampleCtl>();
   SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
@@ -1410,9 +1410,9 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
       if ((h->ticket >= rd.count && h->outstanding == 0) || h->arena_fail) break;
       round_resume(ctx, g, rd, st);
     }
-    res.kernel_ms += elapsed(counted);
-    res.launches += rd.nlaunch - counted;
-    res.spilled += h->spilled;
+    rd.pend.kernel_ms += elapsed(counted);
+    rd.pend.launches += rd.nlaunch - counted;
+    rd.pend.spilled += h->spilled;
     if (std::getenv("EIM_DEBUG_TIMELINE") && rd.model == EIM_IC) {
       std::fprintf(stderr, "timeline count=%llu ids_taken_us=%.1f tail_us=%.1f tasks=%llu spilled=%llu kernel_ms=%.3f\n",
                    (unsigned long long)rd.count, (h->t_last_id - h->t_first) * 1e-3, (h->t_end - h->t_last_id) * 1e-3,
@@ -1434,71 +1434,124 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     counted = rd.nlaunch;
     if (h->arena_fail) {  // rare: redo the whole range with a 4x larger table (and task pool)
       if (attempt >= 4 || rd.bits >= 31) fail(EIM_E_NOMEM, "membership table overflow");
-      rd.bits += 2;
+      rd.bits = std::min<uint32_t>(rd.bits + 2, 31);
       rd.qdirty = true;
       round_start(ctx, g, rd, st, false);
       continue;
     }
     rd.waited = true;
   }
+}
+
+// Source elimination with empty sets dropped (R22): after the launch, the
+// roots leave the sets (sizes - 1) and kidx = exclusive scan of the
+// non-empty flags over the whole launch.  Returns the number of non-empty
+// sets of the launch (once per launch; round_finalize reuses it).
+uint64_t round_elim_kept(eim_ctx* ctx, const eim_graph* g, Round& rd) {
+  if (!rd.launched || rd.count == 0) return 0;
+  if ((rd.rflags & (RF_DROP_ROOT | RF_DROP_EMPTY)) != (RF_DROP_ROOT | RF_DROP_EMPTY))
+    fail(EIM_E_STATE, "round_elim_kept on a round that keeps empty sets");
+  round_wait(ctx, g, rd);
+  if (rd.elim_ready) return rd.kept_total;
+  cudaStream_t st = ctx->stream;
+  SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
+  const uint64_t span = rd.count;
+  rd.roots.reserve(span * sizeof(uint32_t), false, st);
+  rd.kidx.reserve((span + 1) * sizeof(uint32_t), false, st);
+  rd.ksizes.reserve(span * sizeof(uint32_t), false, st);
+  uint32_t* roots = rd.roots.as<uint32_t>();
+  uint32_t* kidx = rd.kidx.as<uint32_t>();
+  roots_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(rd.first, span, g->view.n, philox_key(rd.seed), roots);
+  EIM_CUDA(cudaGetLastError());
+  drop_root_sizes_kernel<<<grid_for(ctx, span + 1, 256), 256, 0, st>>>(rd.sizes.as<uint32_t>(), span, kidx);
+  EIM_CUDA(cudaGetLastError());
+  size_t tmp = 0;
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, kidx, kidx, span + 1, st));
+  ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, kidx, kidx, span + 1, st));
+  ctx->kernel_launches += 3;
+  uint32_t* h32 = reinterpret_cast<uint32_t*>(&h->consumed);
+  EIM_CUDA(cudaMemcpyAsync(h32, kidx + span, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+  rd.kept_total = *h32;
+  rd.elim_ready = true;
+  return rd.kept_total;
+}
+
+SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from, bool keep,
+                            bool consume_all) {
+  SampleResult res;
+  if (!rd.launched || rd.count == 0) return res;
+  if (use > rd.count || from > use) fail(EIM_E_STATE, "round_finalize beyond the launched range");
+  if (from > 0 && (rd.rflags & RF_DROP_ROOT)) fail(EIM_E_STATE, "partial appends of an eliminating round");
+  cudaStream_t st = ctx->stream;
+  SampleCtl* ctl = rd.ctl.as<SampleCtl>();
+  SampleCtl* h = static_cast<SampleCtl*>(ctx->h_pinned);
+  const bool drop_root = (rd.rflags & RF_DROP_ROOT) != 0;
+  const bool drop_empty = drop_root && (rd.rflags & RF_DROP_EMPTY) != 0;
+  if (drop_empty) round_elim_kept(ctx, g, rd);
+  else round_wait(ctx, g, rd);
+  res.kernel_ms = rd.pend.kernel_ms;
+  res.launches = rd.pend.launches;
+  res.spilled = rd.pend.spilled;
+  rd.pend = SampleResult{};
   // ---- append the sets of s_local in [from, use); with keep the round's
   // table stays for a later append of the rest
   if (!keep) {
     rd.launched = false;
     rd.waited = false;
+    rd.elim_ready = false;
   }
   res.kept = res.consumed = use - from;
-  if (use == from) return res;
-  const bool drop_root = (rd.rflags & RF_DROP_ROOT) != 0;
-  const bool drop_empty = drop_root && (rd.rflags & RF_DROP_EMPTY) != 0;
+  if (drop_empty) {
+    // nothing kept and nothing consumed (a rank past the cut of a multi-rank round)
+    if (use == 0 && !consume_all) {
+      res.consumed = 0;
+      return res;
+    }
+    if (consume_all && use != rd.kept_total) fail(EIM_E_STATE, "consume_all needs every non-empty set kept");
+  } else if (use == from) {
+    return res;
+  }
   uint32_t* sizes = rd.sizes.as<uint32_t>() + from;
   uint32_t* roots = nullptr;
   uint32_t* kidx = nullptr;
   uint64_t consumed = use, nsets = use - from;
   size_t tmp = 0, tmp2 = 0;
-  if (drop_root) {
-    // ---- source elimination (R22): roots out of the sets; with drop_empty
-    // only the first `use` non-empty sets are kept and the ids up to the
-    // last kept one are consumed.
-    const uint64_t span = drop_empty ? rd.count : use;
-    rd.roots.reserve(span * sizeof(uint32_t), false, st);
+  if (drop_empty) {
+    // ---- source elimination (R22): only the first `use` non-empty sets are
+    // kept and the ids up to the last kept one are consumed (round_elim_kept
+    // has dropped the roots from the sizes and scanned the non-empty flags).
     roots = rd.roots.as<uint32_t>();
-    roots_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(rd.first, span, g->view.n, philox_key(rd.seed), roots);
-    EIM_CUDA(cudaGetLastError());
-    if (drop_empty) {
-      rd.kidx.reserve((span + 1) * sizeof(uint32_t), false, st);
-      rd.ksizes.reserve(span * sizeof(uint32_t), false, st);
-      kidx = rd.kidx.as<uint32_t>();
+    kidx = rd.kidx.as<uint32_t>();
+    const uint64_t span = rd.count;
+    const uint64_t kept_total = rd.kept_total;
+    consumed = span;
+    nsets = kept_total;
+    if (kept_total >= use && !consume_all) {
+      nsets = use;
+      find_consumed_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(kidx, span, (uint32_t)use, &ctl->consumed);
+      EIM_CUDA(cudaGetLastError());
+      EIM_CUDA(cudaMemcpyAsync(&h->consumed, &ctl->consumed, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+      EIM_CUDA(cudaStreamSynchronize(st));
+      consumed = h->consumed;
+      ctx->kernel_launches += 1;
     }
-    drop_root_sizes_kernel<<<grid_for(ctx, span + 1, 256), 256, 0, st>>>(sizes, span, kidx);
+    if (nsets)
+      compact_sizes_kernel<<<grid_for(ctx, consumed, 256), 256, 0, st>>>(sizes, kidx, consumed,
+                                                                        rd.ksizes.as<uint32_t>());
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches += 1;
+    sizes = rd.ksizes.as<uint32_t>();
+  } else if (drop_root) {
+    // ---- source elimination without dropping sets (eim_sample_rrr_ex)
+    rd.roots.reserve(use * sizeof(uint32_t), false, st);
+    roots = rd.roots.as<uint32_t>();
+    roots_kernel<<<grid_for(ctx, use, 256), 256, 0, st>>>(rd.first, use, g->view.n, philox_key(rd.seed), roots);
+    EIM_CUDA(cudaGetLastError());
+    drop_root_sizes_kernel<<<grid_for(ctx, use + 1, 256), 256, 0, st>>>(sizes, use, nullptr);
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches += 2;
-    if (drop_empty) {
-      EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, kidx, kidx, span + 1, st));
-      ctx->scratch.reserve(std::max<size_t>(tmp, 1 << 20), false, st);
-      EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, kidx, kidx, span + 1, st));
-      uint32_t* h32 = reinterpret_cast<uint32_t*>(&h->consumed);
-      EIM_CUDA(cudaMemcpyAsync(h32, kidx + span, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-      EIM_CUDA(cudaStreamSynchronize(st));
-      const uint64_t kept_total = *h32;
-      consumed = span;
-      nsets = kept_total;
-      if (kept_total >= use) {
-        nsets = use;
-        find_consumed_kernel<<<grid_for(ctx, span, 256), 256, 0, st>>>(kidx, span, (uint32_t)use, &ctl->consumed);
-        EIM_CUDA(cudaGetLastError());
-        EIM_CUDA(cudaMemcpyAsync(&h->consumed, &ctl->consumed, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-        EIM_CUDA(cudaStreamSynchronize(st));
-        consumed = h->consumed;
-        ctx->kernel_launches += 1;
-      }
-      if (nsets)
-        compact_sizes_kernel<<<grid_for(ctx, consumed, 256), 256, 0, st>>>(sizes, kidx, consumed,
-                                                                          rd.ksizes.as<uint32_t>());
-      EIM_CUDA(cudaGetLastError());
-      ctx->kernel_launches += 2;
-      sizes = rd.ksizes.as<uint32_t>();
-    }
   }
   res.kept = nsets;
   res.consumed = consumed - from;

@@ -85,3 +85,14 @@ def test_shard_ranges_partition(first, count, world):
     assert max(sizes) - min(sizes) <= 1
     with pytest.raises(eim.EimError):
         eim.eim_shard_range(0, 10, world, world)
+
+
+def test_create_group_argument_checks():
+    for devs in ([], [-1], [0, -2]):
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_create_group(devs)
+        assert ei.value.status == eim.EIM_E_INVAL
+    if not _has_gpu():
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_create_group([0, 0])
+        assert ei.value.status == eim.EIM_E_CUDA

@@ -22,12 +22,14 @@ for val in values * 2:
     else:
         os.environ[var] = val
     eim.eim_imm_run(ctx, g, c["k"], c["eps"], c["ell"], c["model"], 1)
-    tot, ker = [], []
+    tot, ker, sel = [], [], []
     for _ in range(reps):
         seeds, theta, spread, st = eim.eim_imm_run(ctx, g, c["k"], c["eps"], c["ell"], c["model"], 1)
         tot.append(st["ms_total"])
         ker.append(st["ms_sample_kernel"])
+        sel.append(st["ms_select"])
     ref = ref or seeds.tolist()
     assert seeds.tolist() == ref
-    print(f"{cfg} {var}={val:>6s} imm_ms={statistics.median(tot):8.3f} sample_kernel_ms={statistics.median(ker):8.3f}",
+    print(f"{cfg} {var}={val:>6s} imm_ms={statistics.median(tot):8.3f} sample_kernel_ms={statistics.median(ker):8.3f} "
+          f"select_ms={statistics.median(sel):8.3f}",
           flush=True)
