@@ -500,7 +500,7 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
                                              unsigned char* smem, int gi, uint32_t s_local, bool root,
                                              unsigned long long poff, uint32_t nseed, uint32_t W, int gtid,
                                              uint32_t& found, uint32_t spill_quads, uint32_t task_quads,
-                                             uint32_t help_min, bool& split_any) {
+                                             uint32_t help_min, uint32_t probe_quads, bool& split_any) {
   const SG<G> me = sg_at<G>(smem, gi, W);
   GroupCtl& gc = *me.gc;
   GroupRows<G>& rw = *me.rw;
@@ -565,7 +565,14 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
       tail = head + W;
     }
     uint32_t npieces = 1;
-    if (spill_quads && swept >= spill_quads && tail - head >= 2) {
+    // probe-first rounds: a root traversal that has swept probe_quads quads
+    // is suspended -- its whole backlog leaves as tasks, run after every id
+    // of the round has been probed -- so the heavy samples of a round all
+    // continue from the start of the round's tail phase instead of starting
+    // whenever their id comes up (longest-processing-time order without
+    // knowing the sizes in advance)
+    const bool suspend = root && probe_quads && swept >= probe_quads && tail > head;
+    if (suspend || (spill_quads && swept >= spill_quads && tail - head >= 2)) {
       // quads of the backlog (rows are in rr) -> number of pieces
       const uint32_t B = tail - head;
       uint32_t q = 0;
@@ -578,13 +585,16 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
 #pragma unroll
       for (int i = 0; i < G / 32; ++i) qb += gc.wsum[i];
       npieces = min(B, qb / max(task_quads, 1u));
-      if (npieces < 2) swept = spill_quads / 2;  // look again after a few batches
+      if (suspend) npieces = max(npieces, 1u);
+      else if (npieces < 2) swept = spill_quads / 2;  // look again after a few batches
     }
-    if (npieces >= 2) {
-      // ---- split: keep the first piece of tv vertices, push the rest as tasks of <= tv
+    if (suspend || npieces >= 2) {
+      // ---- split: keep the first piece of tv vertices (none when suspended),
+      // push the rest as tasks of <= tv
       const uint32_t B = tail - head;
       const uint32_t tv = (B + npieces - 1) / npieces;
-      const uint32_t npush = B - tv;
+      const uint32_t keep = suspend ? 0u : tv;
+      const uint32_t npush = B - keep;
       const uint32_t ntasks = (npush + tv - 1) / tv;
       gsync<G>(gi);  // every thread has read wsum
       if (gtid == 0) {
@@ -598,7 +608,7 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
       const unsigned long long po = gc.base, qi = gc.h, tq = R.tcap / TQ, ti = home_queue() * tq + qi;
       const bool ok = po + npush <= R.pcap;
       if (ok)
-        for (uint32_t i = gtid; i < npush; i += G) R.pool[po + i] = me.ring[(head + tv + i) & (W - 1)];
+        for (uint32_t i = gtid; i < npush; i += G) R.pool[po + i] = me.ring[(head + keep + i) & (W - 1)];
       __threadfence();
       gsync<G>(gi);
       for (uint32_t t = gtid; t < ntasks; t += G) {
@@ -612,10 +622,10 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
           const unsigned long long lost = qi + ntasks > tq ? qi + ntasks - max(qi, tq) : 0;
           if (lost) atomicAdd(&ctl->outstanding, 0ull - lost);
         }
-        gc.tail = head + tv;
+        gc.tail = head + keep;
       }
       extra += npush;
-      tail = head + tv;
+      tail = head + keep;
       swept = 0;
       gsync<G>(gi);
     } else if (tail != *(volatile uint32_t*)&gc.tail) {
@@ -704,9 +714,29 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
 // the heavy samples that bound the round), then a new sample id; idle while
 // work is outstanding elsewhere (a running traversal may still split); exit
 // when every id is taken and nothing is outstanding.
-__device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
+__device__ __forceinline__ bool take_id(SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
+  if (vload(&ctl->ticket) < count) {
+    atomicAdd(&ctl->outstanding, 1ull);  // before the ticket: an observer never sees "all taken, none outstanding" early
+    const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
+    if (t == 0) ctl->t_first = gtimer();
+    if (t == count - 1) ctl->t_last_id = gtimer();
+    if (t < count) {
+      gc.s_local = (uint32_t)t;
+      gc.nb = 0;
+      return true;
+    }
+    atomicAdd(&ctl->outstanding, ~0ull);
+  }
+  return false;
+}
+
+// probe_first: new ids before tasks (the tasks are the suspended heavy
+// samples, which then all continue together once every id is taken)
+__device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, uint64_t count, GroupCtl& gc,
+                                           bool probe_first) {
   const volatile unsigned int* cp = R.cancel;
   if (cp[0] || cp[1]) return ACT_EXIT;  // cancelled or paused
+  if (probe_first && take_id(ctl, count, gc)) return ACT_LOCAL;
   const unsigned long long tq = R.tcap / TQ;
   const uint32_t home = home_queue();
   // hint (pushed vs claimed, all queues): scan the queues only when some
@@ -738,18 +768,7 @@ __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, u
       return ACT_TASK;
     }
   }
-  if (vload(&ctl->ticket) < count) {
-    atomicAdd(&ctl->outstanding, 1ull);  // before the ticket: an observer never sees "all taken, none outstanding" early
-    const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
-    if (t == 0) ctl->t_first = gtimer();
-    if (t == count - 1) ctl->t_last_id = gtimer();
-    if (t < count) {
-      gc.s_local = (uint32_t)t;
-      gc.nb = 0;
-      return ACT_LOCAL;
-    }
-    atomicAdd(&ctl->outstanding, ~0ull);
-  }
+  if (!probe_first && take_id(ctl, count, gc)) return ACT_LOCAL;
   if (vload(&ctl->arena_fail)) return ACT_EXIT;  // the host redoes the round
   if (vload(&ctl->outstanding) == 0ull) {
     atomicMax(&ctl->t_end, gtimer());
@@ -771,7 +790,7 @@ constexpr int ic_min_blocks() {
 template <int G, int NSG, class GV>
 __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV g, RoundView R, uint64_t count, uint32_t W,
                                                       SampleCtl* ctl, uint32_t spill_quads, uint32_t task_quads,
-                                                      uint32_t help_min) {
+                                                      uint32_t help_min, uint32_t probe_quads) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int gi = threadIdx.x / G, gtid = threadIdx.x % G, lane = threadIdx.x & 31;
   const SG<G> me = sg_at<G>(smem_raw, gi, W);
@@ -785,7 +804,7 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV 
   __syncthreads();  // every sub-group's job is initialised before anyone helps
   uint32_t backoff = 256;
   for (;;) {
-    if (gtid == 0) gc.action = decide(R, ctl, count, gc);
+    if (gtid == 0) gc.action = decide(R, ctl, count, gc, probe_quads != 0u);
     gsync<G>(gi);
     const uint32_t act = gc.action;
     if (act == ACT_EXIT) break;
@@ -809,7 +828,8 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV 
       uint32_t found = 0;
       bool split_any = false;
       const uint32_t flag = traverse<G, NSG>(g, R, ctl, smem_raw, gi, s_local, act == ACT_LOCAL, poff, nseed, W,
-                                                   gtid, found, spill_quads, task_quads, help_min, split_any);
+                                                   gtid, found, spill_quads, task_quads, help_min, probe_quads,
+                                                   split_any);
       if (gtid == 0) {
         if (found) atomicAdd(&R.sizes[s_local], found);
         if (split_any && act == ACT_LOCAL) atomicAdd(&ctl->spilled, 1ull);
@@ -1214,6 +1234,10 @@ static uint32_t ring_w() {
 }
 
 static uint32_t help_min() { return env_u32("EIM_HELP_QUADS", 1024); }
+// probe-first rounds (EIM_PROBE_QUADS=0: off): root traversals are suspended
+// after this many swept quads.  C2 (tools/ab_env.py, 2 x 5 IMMs): sampler
+// kernels 9.23 ms off, 9.02 at 256, 8.92 at 1024, 8.93 at 4096 per IMM.
+static uint32_t probe_quads() { return env_u32("EIM_PROBE_QUADS", 1024); }
 
 template <int G, int NSG, class K, class GV>
 static void launch_ic_on(eim_ctx* ctx, K kern, const GV& gv, const RoundView& R, uint64_t count, SampleCtl* ctl,
@@ -1223,8 +1247,10 @@ static void launch_ic_on(eim_ctx* ctx, K kern, const GV& gv, const RoundView& R,
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, G * NSG, smem));
   if (per_sm < 1) fail(EIM_E_CUDA, "sampler does not fit on an SM");
   if (spare_sm_slot && per_sm > 1) per_sm -= 1;
+  per_sm = std::min<int>(per_sm, (int)env_u32("EIM_IC_BLOCKS_SM", 64));  // development: resident groups per SM
   const uint64_t blocks = std::max<uint64_t>(1, (uint64_t)per_sm * ctx->sm_count);
-  kern<<<(uint32_t)blocks, G * NSG, smem, st>>>(gv, R, count, W, ctl, spill_quads(), task_quads(), help_min());
+  kern<<<(uint32_t)blocks, G * NSG, smem, st>>>(gv, R, count, W, ctl, spill_quads(), task_quads(), help_min(),
+                                                probe_quads());
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
 }

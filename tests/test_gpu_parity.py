@@ -80,7 +80,10 @@ def test_sample_rrr_C1_all_ids(eim, ctx, graphs, model):
 SPILL_MODES = {"default": {}, "spill_all": {"EIM_SPILL_QUADS": "1", "EIM_TASK_QUADS": "1", "EIM_RING_W": "64"},
                "ring32": {"EIM_SPILL_QUADS": "0", "EIM_RING_W": "32"},
                # general Philox path (the hoisted edge draws need quad ids < 2^32)
-               "nohoist": {"EIM_NO_HOIST": "1"}}
+               "nohoist": {"EIM_NO_HOIST": "1"},
+               # probe-first rounds: nearly every root traversal is suspended into tasks;
+               # and the id-order policy without probing
+               "probe": {"EIM_PROBE_QUADS": "2"}, "noprobe": {"EIM_PROBE_QUADS": "0"}}
 
 
 @pytest.fixture(params=list(SPILL_MODES))
