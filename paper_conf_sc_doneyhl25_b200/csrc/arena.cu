@@ -9,19 +9,50 @@ namespace eim {
 
 namespace {
 
+constexpr unsigned FULL_MASK = 0xFFFFFFFFu;
 
-// One warp per set: C[x] += 1 for every member x (sets have no duplicates).
+// One warp per set: C[x] += d for every member x (sets have no duplicates);
+// d = 1 adds sets [lo, hi) to the histogram, d = -1 removes them.
 __global__ void hist_kernel(const uint32_t* __restrict__ arena, uint32_t ab, const uint64_t* __restrict__ set_start,
                             const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t hi,
-                            uint32_t* __restrict__ C) {
+                            uint32_t* __restrict__ C, uint32_t d) {
   const int lane = threadIdx.x & 31;
   const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t i = lo + warp; i < hi; i += nwarps) {
     const uint64_t st = set_start[i];
     const uint32_t L = set_len[i];
-    for (uint32_t t = lane; t < L; t += 32) atomicAdd(&C[arena_get(arena, st + t, ab)], 1u);
+    for (uint32_t t = lane; t < L; t += 32) atomicAdd(&C[arena_get(arena, st + t, ab)], d);
   }
+}
+
+// Examined in-edges (IC: sum of d^-(v) over the members -- every member was
+// expanded once) or walk steps (LT: |set| - 1, plus the final step unless
+// the walk ended at a vertex without in-edges) of sets [lo, hi).
+__global__ void set_edges_kernel(const uint32_t* __restrict__ arena, uint32_t ab, const uint64_t* __restrict__ set_start,
+                                 const uint32_t* __restrict__ set_len, uint64_t lo, uint64_t hi,
+                                 const uint64_t* __restrict__ off, bool ic, unsigned long long* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  unsigned long long e = 0;
+  for (uint64_t i = lo + warp; i < hi; i += nwarps) {
+    const uint64_t st = set_start[i];
+    const uint32_t L = set_len[i];
+    unsigned long long s = 0;
+    bool sink = false;
+    for (uint32_t t = lane; t < L; t += 32) {
+      const uint32_t v = arena_get(arena, st + t, ab);
+      const uint64_t d = off[v + 1] - off[v];
+      s += d;
+      sink |= d == 0;
+    }
+    const bool any_sink = __any_sync(FULL_MASK, sink);  // i is warp-uniform
+    if (ic) e += s;
+    else if (lane == 0) e += (unsigned long long)L - (any_sink ? 1u : 0u);
+  }
+  for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(FULL_MASK, e, o);
+  if (lane == 0 && e) atomicAdd(out, e);
 }
 
 __global__ void len_to_u64_kernel(const uint32_t* __restrict__ len, uint64_t lo, uint64_t count,
@@ -66,13 +97,35 @@ __global__ void put_kernel(const uint32_t* __restrict__ members, uint64_t total,
 
 }  // namespace
 
-void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi) {
+void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi, int sign) {
   if (hi <= lo) return;
   hist_kernel<<<grid_for(ctx, (hi - lo) * 32, 256), 256, 0, ctx->stream>>>(
       ctx->arena.as<uint32_t>(), ctx->arena_b, ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), lo, hi,
-      ctx->C_total.as<uint32_t>());
+      ctx->C_total.as<uint32_t>(), sign < 0 ? 0xFFFFFFFFu : 1u);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches++;
+}
+
+void drop_sets(eim_ctx* ctx, const eim_graph* g, bool ic, uint64_t keep, uint64_t R, uint64_t* edges) {
+  *edges = 0;
+  if (R <= keep) return;
+  if (!g->view.off) fail(EIM_E_STATE, "drop_sets needs the plain offsets of the graph");
+  cudaStream_t st = ctx->stream;
+  hist_sets(ctx, keep, R, -1);
+  unsigned long long* d = reinterpret_cast<unsigned long long*>(static_cast<char*>(ctx->h_pinned) + 2048);
+  ctx->stage_a.reserve(64, false, st);
+  unsigned long long* dd = ctx->stage_a.as<unsigned long long>();
+  EIM_CUDA(cudaMemsetAsync(dd, 0, sizeof(unsigned long long), st));
+  set_edges_kernel<<<grid_for(ctx, (R - keep) * 32, 256), 256, 0, st>>>(
+      ctx->arena.as<uint32_t>(), ctx->arena_b, ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), keep, R,
+      g->view.off, ic, dd);
+  EIM_CUDA(cudaGetLastError());
+  EIM_CUDA(cudaMemcpyAsync(d, dd, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaMemcpyAsync(d + 1, ctx->set_start.as<uint64_t>() + keep, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaStreamSynchronize(st));
+  ctx->kernel_launches += 2;
+  *edges = d[0];
+  ctx->arena_used = d[1];  // the dropped sets were appended after every kept one
 }
 
 // Compacts sets [lo, lo+count) (set indices) into stage_a (offsets, u64) and

@@ -47,6 +47,18 @@ void DevBuf::release() {
   bytes = 0;
 }
 
+void GreedySlot::release() {
+  DevBuf* b[] = {&C_work, &inv_off, &inv_fill, &inv, &best, &seeds, &gains, &cand, &cidx, &arena_c, &selected, &covered,
+                 &scratch};
+  for (DevBuf* x : b) x->release();
+  if (own_stream && stream) {
+    cudaStreamSynchronize(stream);
+    cudaStreamDestroy(stream);
+  }
+  stream = nullptr;
+  own_stream = false;
+}
+
 }  // namespace eim
 
 using namespace eim;
@@ -88,10 +100,10 @@ eim_status guarded(eim_ctx* ctx, F&& f) {
 bool ctx_ok(const eim_ctx* ctx) { return ctx && ctx->magic == CTX_MAGIC; }
 
 void free_ctx_buffers(eim_ctx* c) {
-  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->covered, &c->ctl, &c->C_total, &c->C_work, &c->inv_off,
-                    &c->inv_fill, &c->inv, &c->best, &c->seeds, &c->gains, &c->scratch, &c->stage_a,
-                    &c->stage_b, &c->stage_c, &c->cand, &c->cidx, &c->arena_c, &c->selected};
+  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->ctl, &c->C_total, &c->C_snap, &c->scratch,
+                    &c->stage_a, &c->stage_b, &c->stage_c};
   for (DevBuf* b : bufs) b->release();
+  for (GreedySlot& g : c->gs) g.release();
   for (Round& r : c->rounds) round_release(r);
 }
 
@@ -139,6 +151,9 @@ eim_ctx* new_ctx(int device, int rank, int world, uint64_t stream, MakeComm&& ma
     EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[0], cudaStreamNonBlocking));
     EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
     EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
+    c->gs[0].stream = c->stream;
+    EIM_CUDA(cudaStreamCreateWithFlags(&c->gs[1].stream, cudaStreamNonBlocking));
+    c->gs[1].own_stream = true;
     EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
     // keep freed stream-ordered memory in the device's pool: reloading a
     // graph or regrowing a buffer reuses it instead of cudaMalloc/cudaFree

@@ -139,6 +139,15 @@ struct Round {
   uint64_t kept_total = 0;    // RF_DROP_EMPTY: non-empty sets of the launch
 };
 
+// Buffers and stream of one greedy NodeSelection (select.cu).  Two slots let
+// the IMM driver run the selections of two rounds concurrently.
+struct GreedySlot {
+  DevBuf C_work, inv_off, inv_fill, inv, best, seeds, gains, cand, cidx, arena_c, selected, covered, scratch;
+  cudaStream_t stream = nullptr;  // slot 0: the context's stream; slot 1: its own
+  bool own_stream = false;
+  void release();
+};
+
 }  // namespace eim
 
 struct eim_graph {
@@ -174,7 +183,7 @@ struct eim_ctx {
   uint64_t kernel_launches;
 
   // arena (persistent, grows)
-  eim::DevBuf arena, set_start, set_len, covered;
+  eim::DevBuf arena, set_start, set_len;
   eim::DevBuf ctl;            // SampleCtl
   eim::Round rounds[2];                         // current + speculative sampler rounds
   cudaStream_t rstream[2] = {};                 // sampler streams of rounds[0], rounds[1]
@@ -183,9 +192,8 @@ struct eim_ctx {
   uint64_t arena_used = 0;                      // arena elements in use (host is the authority)
   uint32_t arena_b = 32;                        // bits per arena element: 32 plain, else log-encoded (R24)
   // per-graph vectors
-  eim::DevBuf C_total, C_work, inv_off, inv_fill, inv;
-  eim::DevBuf best, seeds, gains;
-  eim::DevBuf cand, cidx, arena_c, selected;  // greedy: candidates, remapped arena, picked flags
+  eim::DevBuf C_total, C_snap;                  // coverage counts of R; snapshot for a concurrent selection
+  eim::GreedySlot gs[2];                        // greedy NodeSelection slots
   eim::DevBuf scratch;        // CUB temp storage
   eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
   void* h_pinned = nullptr;   // small pinned host scratch
@@ -253,17 +261,27 @@ uint64_t arena_cursor(eim_ctx* ctx);
 // ---- arena.cu
 // canonical export: offsets (count+1, device u64) + members (device u32), sets ascending
 uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members);
-// histogram of sets [lo, hi) into C_total
-void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi);
+// histogram of sets [lo, hi) into C_total (sign -1: out of it)
+void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi, int sign = 1);
+// Remove the last sets [keep, R) of a plain (32-bit) arena: out of C_total
+// and the arena; *edges = their examined edges (IC) / walk steps (LT).
+void drop_sets(eim_ctx* ctx, const eim_graph* g, bool ic, uint64_t keep, uint64_t R, uint64_t* edges);
 // append externally supplied canonical sets (device pointers) as set ids [base, base+count)
 void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_offsets,
                  const uint32_t* d_members, uint64_t total);
 
 // ---- select.cu
-// Greedy NodeSelection over sets [0, num_sets) with coverage C_total[0..n).
-// Writes seeds/gains (host), returns cov.
+// Greedy NodeSelection over sets [0, num_sets) (arena elements [0, total))
+// with coverage counts C[0..n).  Writes seeds/gains (host), returns cov.
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
                 uint64_t* gains_out);
+// The same, split: enqueue on slot `slot` (its stream waits for the context's
+// stream first), then wait and read the result.  C and the arena prefix must
+// stay unchanged until greedy_collect.  concurrent: another selection runs
+// at the same time (each gets half the SMs).
+void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
+                   uint32_t k, bool concurrent);
+uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out);
 
 // ---- imm.cpp
 void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);

@@ -120,12 +120,12 @@ std::vector<uint64_t> allgather_host(eim_ctx* ctx, Exchange& ex, uint64_t v) {
 // exchanged (exchange_sets), so every rank holds all sets in sample-id order.
 //
 // Lookahead (default on; EIM_NO_LOOKAHEAD=1 turns it off): when the next
-// estimation round adds no more ids than this one, one launch samples both
-// and the next round's sets are appended from the same round table without a
-// launch -- one round tail (the heavy samples' critical paths; for LT the
-// longest walk) instead of two.  Sample ids are fixed labels, so the sets
-// are the same; if the estimation loop stops first the extra sets are
-// discarded.
+// estimation round adds no more ids than this one, or the IMM driver expects
+// it to be needed (next_likely), one launch samples both and the next
+// round's sets are appended from the same round table without a launch --
+// one round tail (the heavy samples' critical paths; for LT the longest
+// walk) instead of two.  Sample ids are fixed labels, so the sets are the
+// same; if the estimation loop stops first the extra sets are discarded.
 //
 // Speculation (opt-in EIM_SPECULATE=1, one GPU): the next round's ids are
 // launched on a second stream right behind the current round's launch and
@@ -159,8 +159,9 @@ class RoundSampler {
     ex_.mem_recv.release();
   }
 
-  // make sets [R, to) final; next_to: the next round's target (lookahead / speculation)
-  void grow(uint64_t& R, uint64_t to, uint64_t next_to) {
+  // make sets [R, to) final; next_to: the next round's target (lookahead /
+  // speculation); next_likely: the next round is expected to be needed
+  void grow(uint64_t& R, uint64_t to, uint64_t next_to, bool next_likely = false) {
     if (to <= R) return;
     const auto t0 = clk::now();
     if (elim_) {
@@ -170,10 +171,13 @@ class RoundSampler {
       grow_speculate(R, to, next_to);
     } else {
       st_->ids_sampled += to - R;
-      grow_shared(R, to, next_to);
+      grow_shared(R, to, next_to, next_likely);
     }
     st_->ms_sample += ms_since(t0);
   }
+
+  // the held lookahead launch can supply sets [from, to) without a launch
+  bool holds(uint64_t from, uint64_t to) const { return held_ && held_done_ == from && launch_end_ >= to; }
 
   void cancel() {
     if (spec_) {
@@ -196,7 +200,7 @@ class RoundSampler {
   // ---- plain runs, any number of ranks.  The held launch covers set
   // indices [launch_first_, launch_end_) (this rank: [my_lo_, my_hi_));
   // sets [launch_first_, held_done_) are appended on every rank.
-  void grow_shared(uint64_t& R, uint64_t to, uint64_t next_to) {
+  void grow_shared(uint64_t& R, uint64_t to, uint64_t next_to, bool next_likely) {
     if (held_) {
       if (held_done_ == R) {
         append_part(R, std::min(launch_end_, to));
@@ -207,7 +211,7 @@ class RoundSampler {
     }
     if (to <= R) return;
     drop_held();
-    const uint64_t end = (lookahead_ && next_to > to && next_to - to <= to - R) ? next_to : to;
+    const uint64_t end = (lookahead_ && next_to > to && (next_to - to <= to - R || next_likely)) ? next_to : to;
     launch_first_ = R;
     launch_end_ = end;
     eim_shard_range(R, end - R, ctx_->rank, W(), &my_lo_, &my_hi_);
@@ -377,31 +381,87 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
   EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
   RoundSampler sampler(ctx, g, model, seed, st, elim);
-  std::vector<uint32_t> S(k);
-  uint64_t R = 0, cov = 0;
+  std::vector<uint32_t> S(k), S_pre(k);
+  uint64_t R = 0, cov = 0, cov_pre = 0;
   uint64_t R_selected = UINT64_MAX;  // |R| the last NodeSelection ran on
+  bool have_pre = false;             // S_pre / cov_pre: NodeSelection on the current R, run ahead
+  // Paired rounds: when one lookahead launch has sampled rounds i and i+1,
+  // both NodeSelections run concurrently (slots 0 and 1, on R_{i+1} and on
+  // R_i with a snapshot of its counts).  If round i's stop test breaks, the
+  // sets of round i+1 that the final phase does not need are dropped again
+  // (drop_sets: counts, arena, examined edges), so every reported number is
+  // the sequential loop's.  One GPU, plain 32-bit arena; EIM_NO_PAIR=1: off.
+  const bool pairing = ctx->world == 1 && !elim && g->view.off && !g->packed && std::getenv("EIM_NO_PAIR") == nullptr;
   double LB = 1.0;
   auto theta_round = [&](uint32_t i) { return (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n); };
   try {
     for (uint32_t i = 1; (double)i < p.log2n; ++i) {
       const uint64_t next = (double)(i + 1) < p.log2n ? theta_round(i + 1) : 0;
-      sampler.grow(R, theta_round(i), next);
-      const auto ts = clk::now();
-      cov = greedy(ctx, n, R, k, S.data(), nullptr);
-      st->ms_select += ms_since(ts);
-      R_selected = R;
+      uint64_t R_sel = R;
+      if (have_pre) {  // this round's selection ran with the previous one
+        have_pre = false;
+        S.swap(S_pre);
+        cov = cov_pre;
+      } else {
+        // round i is expected not to stop the loop when the coverage fraction
+        // of the previous round is below half of what round i needs (the
+        // fraction falls slowly as R grows: C2 0.098, 0.094, 0.090, 0.087,
+        // 0.085); then round i+1 will be needed and is sampled in the same
+        // launch.  A scheduling guess only: the results never depend on it.
+        const bool next_likely = R_selected != UINT64_MAX && R_selected > 0 &&
+                                 (double)cov / (double)R_selected * std::ldexp(1.0, (int)i) < 0.5 * (1.0 + p.eps_p);
+        sampler.grow(R, theta_round(i), next, next_likely);
+        R_sel = R;
+        const auto ts = clk::now();
+        if (pairing && next > R && sampler.holds(R, next)) {
+          const uint64_t total_i = arena_cursor(ctx);
+          ctx->C_snap.reserve((uint64_t)n * sizeof(uint32_t), false, s);
+          EIM_CUDA(cudaMemcpyAsync(ctx->C_snap.p, ctx->C_total.p, (uint64_t)n * sizeof(uint32_t),
+                                   cudaMemcpyDeviceToDevice, s));
+          const auto tg = clk::now();
+          sampler.grow(R, next, 0);  // appends the held sets, no launch
+          st->ms_select -= ms_since(tg);
+          greedy_launch(ctx, 1, n, R_sel, total_i, ctx->C_snap.as<uint32_t>(), k, true);
+          greedy_launch(ctx, 0, n, R, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, true);
+          cov = greedy_collect(ctx, 1, k, S.data(), nullptr);
+          cov_pre = greedy_collect(ctx, 0, k, S_pre.data(), nullptr);
+          have_pre = true;
+        } else {
+          cov = greedy(ctx, n, R, k, S.data(), nullptr);
+        }
+        st->ms_select += ms_since(ts);
+      }
+      R_selected = R_sel;
       if (st->rounds < 64) {
-        st->theta_i[st->rounds] = R;
+        st->theta_i[st->rounds] = R_sel;
         st->cov_i[st->rounds] = cov;
       }
       st->rounds++;
-      if ((double)cov * std::ldexp(1.0, (int)i) >= (1.0 + p.eps_p) * (double)R) {
-        LB = ((double)n * (double)cov) / ((1.0 + p.eps_p) * (double)R);
+      if ((double)cov * std::ldexp(1.0, (int)i) >= (1.0 + p.eps_p) * (double)R_sel) {
+        LB = ((double)n * (double)cov) / ((1.0 + p.eps_p) * (double)R_sel);
         break;
       }
     }
     st->lb = LB;
     const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
+    if (have_pre) {
+      // the loop stopped at round i with the sets of round i+1 appended: keep
+      // max(theta, |R_i|) of them (the sequential loop's final |R|; with a
+      // fresh final phase the estimation phase sampled exactly |R_i|)
+      const uint64_t keep = fresh ? R_selected : std::max<uint64_t>(theta, R_selected);
+      if (keep < R) {
+        uint64_t dropped_edges = 0;
+        drop_sets(ctx, g, model == EIM_IC, keep, R, &dropped_edges);
+        st->edges_examined -= dropped_edges;
+        st->ids_sampled -= R - keep;
+        R = keep;
+      } else {
+        R_selected = R;  // the run-ahead selection is the one on R
+        S.swap(S_pre);
+        cov = cov_pre;
+      }
+      have_pre = false;
+    }
     if (fresh) {  // R23: the final sets are drawn afresh from ids 2^61..
       sampler.restart(EIM_FRESH_BASE);
       arena_reset(ctx, arena_b);

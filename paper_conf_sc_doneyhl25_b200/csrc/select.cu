@@ -237,83 +237,92 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
 
 }  // namespace
 
-uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
-                uint64_t* gains_out) {
-  cudaStream_t st = ctx->stream;
-  const uint64_t total = arena_cursor(ctx);  // arena elements of sets [0, num_sets)
+void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
+                   uint32_t k, bool concurrent) {
+  GreedySlot& S = ctx->gs[slot];
+  cudaStream_t st = S.stream;
+  if (st != ctx->stream) {  // the slot's stream starts after the work enqueued so far (sets, C)
+    EIM_CUDA(cudaEventRecord(ctx->ev0, ctx->stream));
+    EIM_CUDA(cudaStreamWaitEvent(st, ctx->ev0, 0));
+  }
   // ---- 1. candidates (C > 0) in ascending id order; nc stays on the device
   // (buffers are sized for nc <= n), so nothing here waits for the host
-  ctx->inv_fill.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);  // scratch: flags/pos (u32)
-  uint32_t* pos = ctx->inv_fill.as<uint32_t>();
-  flag_kernel<<<grid_for(ctx, (uint64_t)n + 1, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), n, pos);
+  S.inv_fill.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);  // scratch: flags/pos (u32)
+  uint32_t* pos = S.inv_fill.as<uint32_t>();
+  flag_kernel<<<grid_for(ctx, (uint64_t)n + 1, 256), 256, 0, st>>>(C, n, pos);
   EIM_CUDA(cudaGetLastError());
   size_t tmp = 0, tmp2 = 0;
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, pos, pos, (uint64_t)n + 1, st));
-  ctx->inv_off.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);
-  uint64_t* inv_off = ctx->inv_off.as<uint64_t>();
+  S.inv_off.reserve(((uint64_t)n + 1) * sizeof(uint64_t), false, st);
+  uint64_t* inv_off = S.inv_off.as<uint64_t>();
   EIM_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
-  ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
-  EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, pos, pos, (uint64_t)n + 1, st));
-  ctx->cand.reserve((uint64_t)std::max(n, 1u) * 4, false, st);
-  ctx->cidx.reserve((uint64_t)n * 4, false, st);
-  ctx->C_work.reserve(((uint64_t)n + 4) * 4, false, st);
-  compact_kernel<<<grid_for(ctx, n, 256), 256, 0, st>>>(ctx->C_total.as<uint32_t>(), pos, n, ctx->cand.as<uint32_t>(),
-                                                          ctx->cidx.as<uint32_t>(), ctx->C_work.as<uint32_t>(), inv_off);
+  S.scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
+  EIM_CUDA(cub::DeviceScan::ExclusiveSum(S.scratch.p, tmp, pos, pos, (uint64_t)n + 1, st));
+  S.cand.reserve((uint64_t)std::max(n, 1u) * 4, false, st);
+  S.cidx.reserve((uint64_t)n * 4, false, st);
+  S.C_work.reserve(((uint64_t)n + 4) * 4, false, st);
+  compact_kernel<<<grid_for(ctx, n, 256), 256, 0, st>>>(C, pos, n, S.cand.as<uint32_t>(), S.cidx.as<uint32_t>(),
+                                                          S.C_work.as<uint32_t>(), inv_off);
   EIM_CUDA(cudaGetLastError());
   // ---- 2. arena in candidate indices + inverted index
-  ctx->arena_c.reserve(std::max<uint64_t>(total, 1) * 4, false, st);
+  S.arena_c.reserve(std::max<uint64_t>(total, 1) * 4, false, st);
   if (total)
     remap_kernel<<<grid_for(ctx, total, 256), 256, 0, st>>>(ctx->arena.as<uint32_t>(), ctx->arena_b, total,
-                                                              ctx->cidx.as<uint32_t>(), ctx->arena_c.as<uint32_t>());
-  EIM_CUDA(cub::DeviceScan::InclusiveSum(ctx->scratch.p, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
-  ctx->inv.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
+                                                              S.cidx.as<uint32_t>(), S.arena_c.as<uint32_t>());
+  EIM_CUDA(cub::DeviceScan::InclusiveSum(S.scratch.p, tmp2, inv_off, inv_off, (uint64_t)n + 1, st));
+  S.inv.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
   if (num_sets > 0 && total > 0) {
     invert_kernel<<<grid_for(ctx, num_sets * 32, 256), 256, 0, st>>>(
-        ctx->arena_c.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), num_sets,
-        reinterpret_cast<unsigned long long*>(inv_off), ctx->inv.as<uint32_t>());
+        S.arena_c.as<uint32_t>(), ctx->set_start.as<uint64_t>(), ctx->set_len.as<uint32_t>(), num_sets,
+        reinterpret_cast<unsigned long long*>(inv_off), S.inv.as<uint32_t>());
     EIM_CUDA(cudaGetLastError());
   }
   // ---- 3. the k picks in one cooperative kernel
-  ctx->covered.reserve(std::max<uint64_t>(num_sets, 1), false, st);
-  ctx->selected.reserve((uint64_t)n + 4, false, st);
-  ctx->seeds.reserve((uint64_t)k * sizeof(uint32_t), false, st);
-  ctx->gains.reserve((uint64_t)k * sizeof(unsigned long long), false, st);
-  EIM_CUDA(cudaMemsetAsync(ctx->covered.p, 0, std::max<uint64_t>(num_sets, 1), st));
-  EIM_CUDA(cudaMemsetAsync(ctx->selected.p, 0, (uint64_t)n + 4, st));
+  S.covered.reserve(std::max<uint64_t>(num_sets, 1), false, st);
+  S.selected.reserve((uint64_t)n + 4, false, st);
+  S.seeds.reserve((uint64_t)k * sizeof(uint32_t), false, st);
+  S.gains.reserve((uint64_t)k * sizeof(unsigned long long), false, st);
+  EIM_CUDA(cudaMemsetAsync(S.covered.p, 0, std::max<uint64_t>(num_sets, 1), st));
+  EIM_CUDA(cudaMemsetAsync(S.selected.p, 0, (uint64_t)n + 4, st));
   int per_sm = 0;
   EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
   const char* gbe = getenv("EIM_GREEDY_BLOCKS");  // development: grid of the greedy kernel
   uint32_t blocks = gbe ? (uint32_t)atoi(gbe) : (uint32_t)ctx->sm_count;
+  // two concurrent selections get half the SMs each: measured on C3 (both
+  // selections of the paired rounds 1 and 2), 74 + 74 blocks take 1.33 ms
+  // against 1.93 ms for the two one after the other on 148 blocks, while
+  // two 148-block grids launched together take 2.0 ms (they do not overlap)
+  if (concurrent) blocks = std::max(1u, blocks / 2);
   blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
-  ctx->best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
-  uint32_t* zc = reinterpret_cast<uint32_t*>(ctx->best.as<unsigned long long>() + blocks);
+  S.best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
+  uint32_t* zc = reinterpret_cast<uint32_t*>(S.best.as<unsigned long long>() + blocks);
   EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
   GreedyArgs a;
   a.k = k;
   a.nc = pos + n;
-  a.W = ctx->C_work.as<uint32_t>();
-  a.cand = ctx->cand.as<uint32_t>();
+  a.W = S.C_work.as<uint32_t>();
+  a.cand = S.cand.as<uint32_t>();
   a.inv_off = inv_off;
-  a.inv = ctx->inv.as<uint32_t>();
-  a.F = ctx->covered.as<uint8_t>();
+  a.inv = S.inv.as<uint32_t>();
+  a.F = S.covered.as<uint8_t>();
   a.set_start = ctx->set_start.as<uint64_t>();
   a.set_len = ctx->set_len.as<uint32_t>();
-  a.arena_c = ctx->arena_c.as<uint32_t>();
-  a.blockmax = ctx->best.as<unsigned long long>();
-  a.selected = ctx->selected.as<uint8_t>();
+  a.arena_c = S.arena_c.as<uint32_t>();
+  a.blockmax = S.best.as<unsigned long long>();
+  a.selected = S.selected.as<uint8_t>();
   a.zc = zc;
-  a.seeds = ctx->seeds.as<uint32_t>();
-  a.gains = ctx->gains.as<unsigned long long>();
+  a.seeds = S.seeds.as<uint32_t>();
+  a.gains = S.gains.as<unsigned long long>();
   a.dbg = nullptr;
   const char* gdbg = getenv("EIM_DEBUG_GREEDY");
-  if (gdbg) {
+  if (gdbg && slot == 0) {
     ctx->stage_a.reserve((uint64_t)k * 24 + 64, false, st);
     a.dbg = ctx->stage_a.as<unsigned long long>();
   }
   void* args[] = {&a};
   EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
   ctx->kernel_launches += 9;
-  if (gdbg) {
+  if (a.dbg) {
     std::vector<unsigned long long> hd((size_t)k * 3);
     EIM_CUDA(cudaMemcpyAsync(hd.data(), a.dbg, (size_t)k * 24, cudaMemcpyDeviceToHost, st));
     EIM_CUDA(cudaStreamSynchronize(st));
@@ -323,16 +332,31 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
       fclose(f);
     }
   }
+}
+
+uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out) {
+  GreedySlot& S = ctx->gs[slot];
+  cudaStream_t st = S.stream;
   std::vector<unsigned long long> g(k);
-  EIM_CUDA(cudaMemcpyAsync(seeds_out, ctx->seeds.p, (uint64_t)k * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-  EIM_CUDA(cudaMemcpyAsync(g.data(), ctx->gains.p, (uint64_t)k * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaMemcpyAsync(seeds_out, S.seeds.p, (uint64_t)k * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+  EIM_CUDA(cudaMemcpyAsync(g.data(), S.gains.p, (uint64_t)k * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
+  if (st != ctx->stream) {  // later work on the context's stream may reuse what the selection read
+    EIM_CUDA(cudaEventRecord(ctx->ev1, st));
+    EIM_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->ev1, 0));
+  }
   uint64_t cov = 0;
   for (uint32_t j = 0; j < k; ++j) {
     cov += g[j];
     if (gains_out) gains_out[j] = g[j];
   }
   return cov;
+}
+
+uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
+                uint64_t* gains_out) {
+  greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, false);
+  return greedy_collect(ctx, 0, k, seeds_out, gains_out);
 }
 
 }  // namespace eim
