@@ -38,18 +38,38 @@ PHILOX_PROBE = os.path.join(ROOT, "tools", "philox_roof", "philox_roof")
 
 
 def philox_roof_gwords():
+    """(peak Gwords/s, source, probe lines): the probe output rides along in
+    the bench line (roofline.peak_probe), so the peak used is on record."""
     try:
         out = subprocess.run([PHILOX_PROBE], capture_output=True, text=True, timeout=60).stdout
-        vals = [json.loads(l)["words_per_s"] for l in out.splitlines() if l.startswith("{")]
-        if vals:
-            return max(vals) / 1e9, "measured live (tools/philox_roof)"
+        lines = [json.loads(l) for l in out.splitlines() if l.startswith("{")]
+        if lines:
+            return max(l["words_per_s"] for l in lines) / 1e9, "measured live (tools/philox_roof)", lines
     except Exception:
         pass
     try:
         with open(os.path.join(ROOT, "profiles", "philox_roof.json")) as f:
-            return json.load(f)["roof_words_per_s"] / 1e9, "profiles/philox_roof.json (earlier measurement)"
+            return json.load(f)["roof_words_per_s"] / 1e9, "profiles/philox_roof.json (earlier measurement)", []
     except Exception:
-        return 1630.0, "fallback constant"
+        return 1630.0, "fallback constant", []
+
+
+def ncu_traffic(model):
+    """DRAM bytes per launch of the dominant kernel from the newest committed
+    `ncu --set full` summary of this round (profiles/r02_*), else round 1's."""
+    names = (["r02_ncu_ic_kernel.json", "ncu_sampler.json"] if model == "IC" else
+             ["r02_ncu_lt_aug_kernel.json", "ncu_sampler_lt.json"])
+    for nm in names:
+        path = os.path.join(ROOT, "profiles", nm)
+        if not os.path.exists(path):
+            continue
+        try:
+            ls = [l for l in json.load(open(path))["launches"] if "dram_bytes" in l]
+            if ls:
+                return sum(l["dram_bytes"] for l in ls) / len(ls), f"profiles/{nm}"
+        except Exception:
+            continue
+    return None, None
 
 
 def _peaks():
@@ -117,7 +137,10 @@ class ClockSampler:
 
 
 def run_reference(args):
-    """The oracle (CPU, as it stands) on bounded samples of the same workload."""
+    """The reference arm: the CPU oracle as it stands, one full IMM of the same
+    workload per step (same metric: theta / IMM seconds).  Warm-up steps only
+    page the graph in (a 64-id oracle sample each): the oracle keeps no state
+    between calls, so a warm-up IMM would measure nothing new."""
     import inputs
     import oracle
     rank = int(os.environ.get("RANK", "0"))
@@ -126,21 +149,25 @@ def run_reference(args):
     c = inputs.CONFIGS[args.config]
     off, nbr = inputs.config_graph(args.config, seed=GRAPH_SEED)
     cores = max(1, min(64, os.cpu_count() or 1))
-    block = 256 * cores
     for w in range(args.warmup):
-        oracle.sample(off, nbr, c["model"], RUN_SEED, w * block, block, nthreads=cores)
-    t0 = time.perf_counter()
-    for s in range(args.steps):
-        oracle.sample(off, nbr, c["model"], RUN_SEED, (args.warmup + s) * block, block, nthreads=cores)
-    dt = time.perf_counter() - t0
-    v = args.steps * block / dt
+        oracle.sample(off, nbr, c["model"], RUN_SEED, w * 64, 64, nthreads=cores)
+    times, theta = [], None
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        r = oracle.imm(off, nbr, c["k"], c["eps"], c["ell"], c["model"], RUN_SEED, nthreads=cores)
+        times.append(time.perf_counter() - t0)
+        theta = r["theta"]
+    dt = sum(times)
+    v = args.steps * theta / dt
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": "u32", "data": "synthetic", "config": {"workload": workload_desc(args.config)},
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": workload_desc(args.config), "theta": theta},
+        "imm_s": dt / args.steps,
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
-                         "sample": f"per step: oracle RRR sampling of {block} consecutive sample ids of the workload "
-                                   f"on {cores} threads (greedy excluded)"},
+                         "sample": f"per step: one full oracle IMM run of the workload (theta={theta}; sampling on "
+                                   f"{cores} threads, greedy single-threaded), the same work as the GPU arm's step"},
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -169,8 +196,8 @@ def main():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
-    ap.add_argument("--budget-ids", type=int, default=1 << 20,
-                    help="fixed sample budget of the sampler-throughput leg (0: skip)")
+    ap.add_argument("--budget-ids", type=int, default=1 << 24,
+                    help="fixed sample budget of the sampler-throughput leg, SURVEY 8(d): ids [0, 2^24) (0: skip)")
     ap.add_argument("--variant-steps", type=int, default=3,
                     help="timed steps of each NEXT-row variant (log-encoded store, source elimination, "
                          "fresh final phase); 0: skip")
@@ -246,8 +273,9 @@ def main():
     k_ms = sum(s["ms_sample_kernel"] for s in stats)
     k_launch = sum(s["sample_launches"] for s in stats)
     k_edges_local = sum(s["edges_examined"] for s in stats)
+    probe = []
     if c["model"] == "IC":
-        peak, peak_src = philox_roof_gwords() if rank == 0 else (1630.0, "")
+        peak, peak_src, probe = philox_roof_gwords() if rank == 0 else (1630.0, "", [])
         achieved = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
     else:
         # LT walk step on the walk store: one 16-B entry (v, d(v), off[v]) + one
@@ -255,14 +283,16 @@ def main():
         peak = float(_peaks().get("hbm_gbs", 8000.0))
         peak_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in _peaks() else "fallback 8 TB/s"
         achieved = (LT_STEP_BYTES * k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
-    traffic = None  # DRAM bytes per sampler launch from the committed ncu --set full capture
-    tpath = os.path.join(ROOT, "profiles", "ncu_sampler.json" if c["model"] == "IC" else "ncu_sampler_lt.json")
-    if os.path.exists(tpath):
-        try:
-            ls = [l for l in json.load(open(tpath))["launches"] if "dram_bytes" in l]
-            traffic = sum(l["dram_bytes"] for l in ls) / len(ls) if ls else None
-        except Exception:
-            traffic = None
+    traffic, traffic_src = ncu_traffic(c["model"])  # DRAM bytes per launch, committed ncu --set full capture
+    # the greedy pick kernel: latency-bound (two grid barriers and ~4 dependent
+    # L2 round trips per pick), reported as device time per pick
+    g_ms = sum(s["ms_select_kernel"] for s in stats)
+    g_picks = sum(s["select_picks"] for s in stats)
+    greedy_line = {"kernel": "greedy_kernel (k greedy picks per NodeSelection, cooperative)", "bound": "latency",
+                   "us_per_pick": (g_ms * 1e3 / g_picks) if g_picks else None,
+                   "selections_per_imm": stats[-1]["select_launches"], "picks_per_imm": stats[-1]["select_picks"],
+                   "kernel_ms_per_imm": g_ms / args.steps,
+                   "note": "two concurrent selections (paired rounds) both count their device time"}
 
     # end to end through the public API with host buffers: H2D of the graph
     # from pinned memory + IMM + D2H of the result, every step
@@ -334,8 +364,7 @@ def main():
                 variants[-1]["threshold_stream_frac_hbm"] = gbs / hbm
                 variants[-1]["edges_per_s"] = vst["edges_examined"] / (vst["ms_sample_kernel"] / 1e3)
                 if args.budget_ids > 0:  # the same layout on the fixed sample budget (no round tails)
-                    eim.eim_sample_rrr(ctx, gv, c["model"], RUN_SEED, 0, args.budget_ids)
-                    sb = eim.eim_get_stats(ctx)
+                    sb = eim.eim_sample_rrr_stats(ctx, gv, c["model"], RUN_SEED, 0, args.budget_ids)
                     bgbs = 4.0 * sb["edges_examined"] / (sb["ms_sample_kernel"] / 1e3) / 1e9
                     variants[-1]["fixed_budget"] = {
                         "ids": args.budget_ids, "kernel_ms": sb["ms_sample_kernel"],
@@ -348,8 +377,7 @@ def main():
     if args.budget_ids > 0:
         lo_b, hi_b = eim.eim_shard_range(0, args.budget_ids, rank, world)
         eim.eim_sample_rrr(ctx, g, c["model"], RUN_SEED, lo_b, min(hi_b - lo_b, 4096))  # warm-up
-        eim.eim_sample_rrr(ctx, g, c["model"], RUN_SEED, lo_b, hi_b - lo_b)
-        sb = eim.eim_get_stats(ctx)
+        sb = eim.eim_sample_rrr_stats(ctx, g, c["model"], RUN_SEED, lo_b, hi_b - lo_b)
         bt = torch.tensor([sb["ms_sample_kernel"], float(sb["edges_examined"])], dtype=torch.float64, device=dev)
         if world > 1:
             bmax = bt[:1].clone()
@@ -383,18 +411,20 @@ def main():
             "sampler_sets_per_s": theta_all / (sum(s["ms_sample"] for s in stats) / args.steps / 1e3),
             "phase_ms": {"sample": sum(s["ms_sample"] for s in stats) / args.steps,
                          "sample_kernel": k_ms / args.steps,
+                         "select_kernel": g_ms / args.steps,
                          "select": sum(s["ms_select"] for s in stats) / args.steps,
                          "comm": sum(s["ms_comm"] for s in stats) / args.steps},
             "roofline": ({"bound": "alu", "kernel": "ic_kernel (IC sampler, incl. split-off tasks)", "achieved": achieved,
                           "peak": peak, "unit": "Gedge/s", "frac": (achieved / peak) if achieved else None,
-                          "traffic": traffic,
+                          "traffic": traffic, "traffic_source": traffic_src,
                           "peak_basis": "Philox4x32-10 word rate of this GPU (one word per examined in-edge; best of the "
                                         "plain and the sampler's hoisted form, tools/philox_roof), "
-                                        + peak_src + "; DESIGN.md §6"} if c["model"] == "IC" else
+                                        + peak_src + "; DESIGN.md §6", "peak_probe": probe} if c["model"] == "IC" else
                          {"bound": "hbm", "kernel": "lt_aug_kernel (LT reverse walks on the walk store)", "achieved": achieved,
                           "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
-                          "traffic": traffic,
+                          "traffic": traffic, "traffic_source": traffic_src,
                           "peak_basis": f"{LT_STEP_BYTES:.0f} algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
+            "greedy": greedy_line,
             # IC: examined edges/s vs the Philox roof; LT: LT_STEP_BYTES per walk step vs HBM
             "sampler_fixed_budget": (dict(budget, frac=(budget["edges_per_s"] / 1e9 / world / peak)
                                           if c["model"] == "IC" else

@@ -69,6 +69,10 @@ typedef struct {
   double ms_sample_kernel;      /* device time of the sampler kernels (CUDA events on the ctx stream) */
   uint64_t ids_sampled;         /* sample ids drawn by the run, all ranks (> theta with EIM_F_SOURCE_ELIM) */
   uint64_t arena_bytes;         /* device bytes of the stored sets R (log-encoded with an EIM_G_LOG_ENCODE graph) */
+  double ms_select_kernel;      /* device time of the greedy pick kernels (CUDA events on their streams; two
+                                   concurrent selections both count) */
+  uint32_t select_launches;     /* greedy NodeSelections run */
+  uint64_t select_picks;        /* greedy picks over all NodeSelections (k per selection) */
 } eim_stats;
 
 /* Run flags of eim_imm_run_ex / eim_sample_rrr_ex. */
@@ -201,8 +205,11 @@ eim_status eim_graph_bytes(const eim_graph* g, uint64_t* bytes);
  * EIM_F_SOURCE_ELIM: the first theta non-empty sets in sample-id order,
  * wherever the cut falls).  stats_out->edges_examined, spilled_samples,
  * sample_launches and the ms_* fields are this rank's.
- * Errors: EIM_E_INVAL, EIM_E_STATE (graph from another ctx / freed),
+ * Errors: EIM_E_INVAL (also when theta = ceil(lambda* / LB) would exceed
+ * 2^32 - 1 sets), EIM_E_STATE (graph from another ctx / freed),
  * EIM_E_NOMEM, EIM_E_CUDA, EIM_E_NCCL.
+ * Large theta is sampled in several launches, each sized to keep its
+ * membership table within 8 GiB (the results do not depend on the split).
  */
 eim_status eim_imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell,
                        eim_model model, uint64_t seed, uint32_t* seeds_out, uint64_t* theta_out,
@@ -244,6 +251,8 @@ eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, 
  * seeds_out[k] in pick order; ties go to the lowest vertex id; when every
  * set is covered the remaining picks are the lowest unselected ids (R10).
  * gains_out[k] (nullable) = marginal coverage of each pick.
+ * Errors: EIM_E_INVAL for num_sets >= 2^32, decreasing offsets, a member
+ * >= n or a member repeated within a set, k outside [1, n].
  */
 eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const uint64_t* offsets,
                             const uint32_t* members, uint32_t k, uint32_t* seeds_out,

@@ -64,6 +64,9 @@ class Stats(ctypes.Structure):
         ("ms_sample_kernel", ctypes.c_double),
         ("ids_sampled", ctypes.c_uint64),
         ("arena_bytes", ctypes.c_uint64),
+        ("ms_select_kernel", ctypes.c_double),
+        ("select_launches", ctypes.c_uint32),
+        ("select_picks", ctypes.c_uint64),
     ]
 
     def as_dict(self):
@@ -241,6 +244,19 @@ def eim_sample_rrr(ctx, g, model, seed, first_id, count, members_cap=None, flags
             continue
         _check(s, ctx)
         return offsets, members[: int(total.value)]
+
+
+def eim_sample_rrr_stats(ctx, g, model, seed, first_id, count, flags=0):
+    """Samples ids [first_id, first_id+count) and returns the call's stats
+    only (the members stay on the device: members_cap 0 => EIM_E_CAPACITY
+    after the sampling, which is the expected outcome here)."""
+    offsets = np.zeros(count + 1, dtype=np.uint64)
+    total = ctypes.c_uint64()
+    s = lib().eim_sample_rrr_ex(ctx, g, MODELS[model], seed, first_id, count, flags, offsets.ctypes.data, None, 0,
+                                ctypes.addressof(total))
+    if s not in (EIM_OK, EIM_E_CAPACITY):
+        _check(s, ctx)
+    return eim_get_stats(ctx)
 
 
 def eim_select_seeds(ctx, n, offsets, members, k):

@@ -131,7 +131,7 @@ void drop_sets(eim_ctx* ctx, const eim_graph* g, bool ic, uint64_t keep, uint64_
 // Compacts sets [lo, lo+count) (set indices) into stage_a (offsets, u64) and
 // stage_b (members).  Returns the member total.  sort: ascending within sets.
 static uint64_t compact_sets(eim_ctx* ctx, uint64_t lo, uint64_t count, bool sort, uint64_t** d_offsets,
-                             uint32_t** d_members) {
+                             uint32_t** d_members, uint64_t sort_cap = UINT64_MAX) {
   cudaStream_t st = ctx->stream;
   ctx->stage_a.reserve((count + 1) * sizeof(uint64_t), false, st);
   uint64_t* offs = ctx->stage_a.as<uint64_t>();
@@ -145,6 +145,11 @@ static uint64_t compact_sets(eim_ctx* ctx, uint64_t lo, uint64_t count, bool sor
   EIM_CUDA(cudaMemcpyAsync(ctx->h_pinned, offs + count, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   total = *static_cast<uint64_t*>(ctx->h_pinned);
+  if (total > sort_cap) {  // the members are not wanted (capacity exceeded): offsets only
+    *d_offsets = offs;
+    *d_members = nullptr;
+    return total;
+  }
   ctx->stage_b.reserve(std::max<uint64_t>(total, 1) * sizeof(uint32_t), false, st);
   uint32_t* out = ctx->stage_b.as<uint32_t>();
   if (count > 0) {
@@ -174,8 +179,9 @@ static uint64_t compact_sets(eim_ctx* ctx, uint64_t lo, uint64_t count, bool sor
   return total;
 }
 
-uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members) {
-  return compact_sets(ctx, 0, count, true, d_offsets, d_members);
+uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members, uint64_t members_cap) {
+  // members that will not be copied out (more than members_cap) need no sort
+  return compact_sets(ctx, 0, count, true, d_offsets, d_members, members_cap);
 }
 
 uint64_t compact_range(eim_ctx* ctx, uint64_t lo, uint64_t count, uint64_t** d_offsets, uint32_t** d_members) {

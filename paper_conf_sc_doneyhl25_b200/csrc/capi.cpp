@@ -3,6 +3,7 @@
 #include <chrono>
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "eim_internal.h"
 
@@ -51,6 +52,10 @@ void GreedySlot::release() {
   DevBuf* b[] = {&C_work, &inv_off, &inv_fill, &inv, &best, &seeds, &gains, &cand, &cidx, &arena_c, &selected, &covered,
                  &scratch};
   for (DevBuf* x : b) x->release();
+  for (cudaEvent_t& e : ev) {
+    if (e) cudaEventDestroy(e);
+    e = nullptr;
+  }
   if (own_stream && stream) {
     cudaStreamSynchronize(stream);
     cudaStreamDestroy(stream);
@@ -399,7 +404,7 @@ eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, 
     ctx->last_stats.ms_sample = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     uint64_t* d_off = nullptr;
     uint32_t* d_mem = nullptr;
-    const uint64_t total = export_sets(ctx, count, &d_off, &d_mem);
+    const uint64_t total = export_sets(ctx, count, &d_off, &d_mem, members_cap);
     *members_total = total;
     EIM_CUDA(cudaMemcpyAsync(offsets_out, d_off, (count + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
     if (total > members_cap) {
@@ -430,10 +435,19 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     if (offsets[0] != 0) fail(EIM_E_INVAL, "offsets[0] != 0");
     for (uint64_t i = 0; i < num_sets; ++i)
       if (offsets[i + 1] < offsets[i]) fail(EIM_E_INVAL, "offsets not non-decreasing");
+    if (num_sets >= (1ull << 32)) fail(EIM_E_INVAL, "at most 2^32 - 1 sets");
     const uint64_t total = offsets[num_sets];
     if (total && !members) fail(EIM_E_INVAL, "members is NULL");
-    for (uint64_t i = 0; i < total; ++i)
-      if (members[i] >= n) fail(EIM_E_INVAL, "member id >= n");
+    // members < n and distinct within each set (a duplicate would count a
+    // set twice in C and corrupt the gains): stamp[v] = last set index + 1
+    std::vector<uint32_t> stamp(n, 0u);
+    for (uint64_t i = 0; i < num_sets; ++i)
+      for (uint64_t j = offsets[i]; j < offsets[i + 1]; ++j) {
+        const uint32_t v = members[j];
+        if (v >= n) fail(EIM_E_INVAL, "member id >= n");
+        if (stamp[v] == (uint32_t)(i + 1)) fail(EIM_E_INVAL, "duplicate member within a set");
+        stamp[v] = (uint32_t)(i + 1);
+      }
     cudaStream_t st = ctx->stream;
     ctx->cov_n = 0;
     arena_reset(ctx);
@@ -446,8 +460,12 @@ eim_status eim_select_seeds(eim_ctx* ctx, uint32_t n, uint64_t num_sets, const u
     append_sets(ctx, 0, num_sets, ctx->stage_a.as<uint64_t>(), ctx->stage_b.as<uint32_t>(), total);
     hist_sets(ctx, 0, num_sets);
     const auto t0 = std::chrono::steady_clock::now();
-    const uint64_t cov = greedy(ctx, n, num_sets, k, seeds_out, gains_out);
+    double kms = 0;
+    const uint64_t cov = greedy(ctx, n, num_sets, k, seeds_out, gains_out, &kms);
     std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
+    ctx->last_stats.ms_select_kernel = kms;
+    ctx->last_stats.select_launches = 1;
+    ctx->last_stats.select_picks = k;
     ctx->last_stats.cov = cov;
     ctx->last_stats.theta = num_sets;
     ctx->last_stats.arena_elems = total;

@@ -145,6 +145,7 @@ struct GreedySlot {
   DevBuf C_work, inv_off, inv_fill, inv, best, seeds, gains, cand, cidx, arena_c, selected, covered, scratch;
   cudaStream_t stream = nullptr;  // slot 0: the context's stream; slot 1: its own
   bool own_stream = false;
+  cudaEvent_t ev[2] = {};          // around the pick kernel
   void release();
 };
 
@@ -167,6 +168,7 @@ struct eim_graph {
   void* d_cum = nullptr;
   void* d_aug = nullptr;         // LT walk store of the plain graph, built on the first LT run (uint4 per in-edge)
   uint64_t aug_bytes = 0;
+  bool aug_failed = false;       // the walk store did not fit: LT runs on the plain store
   bool lt_ok = true;             // weighted: every row's weights sum to <= 2^32 (LT usable)
   uint64_t bytes = 0;            // device bytes of the store
   int proper_edge = -1;  // has an edge u -> v, u != v (1/0; -1 = not yet computed)
@@ -217,7 +219,11 @@ void graph_attach_weights(eim_ctx* ctx, eim_graph* g, const uint32_t* h_x);
 bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g);
 
 // ---- sample.cu
-// Samples ids [first, first+count) into ctx->arena; set index = id - set_base.
+// Sample ids per launch that keep the round's membership table within its
+// memory budget (from the mean set size of earlier launches).
+uint64_t max_launch_ids(const eim_ctx* ctx);
+// Samples ids [first, first+count) into ctx->arena; set index = id - set_base
+// (in launches of at most max_launch_ids ids).
 // Histogram into C when hist is true.  (= round_launch + round_finalize)
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
                           uint64_t first, uint64_t count, uint64_t set_base, bool hist, uint32_t rflags = 0);
@@ -260,7 +266,10 @@ uint64_t arena_cursor(eim_ctx* ctx);
 
 // ---- arena.cu
 // canonical export: offsets (count+1, device u64) + members (device u32), sets ascending
-uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members);
+// (members are sorted only when the total fits members_cap: otherwise the
+// caller reports EIM_E_CAPACITY and copies none)
+uint64_t export_sets(eim_ctx* ctx, uint64_t count, uint64_t** d_offsets, uint32_t** d_members,
+                     uint64_t members_cap = UINT64_MAX);
 // histogram of sets [lo, hi) into C_total (sign -1: out of it)
 void hist_sets(eim_ctx* ctx, uint64_t lo, uint64_t hi, int sign = 1);
 // Remove the last sets [keep, R) of a plain (32-bit) arena: out of C_total
@@ -274,14 +283,15 @@ void append_sets(eim_ctx* ctx, uint64_t base, uint64_t count, const uint64_t* d_
 // Greedy NodeSelection over sets [0, num_sets) (arena elements [0, total))
 // with coverage counts C[0..n).  Writes seeds/gains (host), returns cov.
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
-                uint64_t* gains_out);
+                uint64_t* gains_out, double* kernel_ms = nullptr);
 // The same, split: enqueue on slot `slot` (its stream waits for the context's
 // stream first), then wait and read the result.  C and the arena prefix must
 // stay unchanged until greedy_collect.  concurrent: another selection runs
 // at the same time (each gets half the SMs).
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
                    uint32_t k, bool concurrent);
-uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out);
+uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
+                        double* kernel_ms = nullptr);
 
 // ---- imm.cpp
 void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);

@@ -94,6 +94,8 @@ void exchange_sets(eim_ctx* ctx, uint64_t a, uint64_t b, const std::vector<std::
   }
   hist_sets(ctx, a, b);
   EIM_CUDA(cudaStreamSynchronize(s));
+  // the same on every rank (the launch sizes of all ranks must agree)
+  ctx->est_mean_size = std::max(1.0, (double)arena_cursor(ctx) / (double)std::max<uint64_t>(b, 1));
   st->ms_comm += ms_since(t0);
 }
 
@@ -211,7 +213,24 @@ class RoundSampler {
     }
     if (to <= R) return;
     drop_held();
-    const uint64_t end = (lookahead_ && next_to > to && (next_to - to <= to - R || next_likely)) ? next_to : to;
+    // launches sized for the membership-table budget: a range above it is
+    // sampled in several launches (sample ids are fixed labels, same sets)
+    const uint64_t cap = max_launch_ids(ctx_) * (uint64_t)W();
+    while (to - R > cap) {
+      launch_range(R, R + cap);
+      append_part(R, R + cap);
+      R += cap;
+    }
+    uint64_t end = (lookahead_ && next_to > to && (next_to - to <= to - R || next_likely)) ? next_to : to;
+    if (end - R > cap) end = to;
+    launch_range(R, end);
+    append_part(R, to);
+    R = to;
+  }
+
+  // Launch this rank's share of the set indices [first, end) and hold it.
+  void launch_range(uint64_t first, uint64_t end) {
+    const uint64_t R = first;
     launch_first_ = R;
     launch_end_ = end;
     eim_shard_range(R, end - R, ctx_->rank, W(), &my_lo_, &my_hi_);
@@ -221,8 +240,6 @@ class RoundSampler {
                    false);
     held_ = true;
     held_done_ = R;
-    append_part(R, to);
-    R = to;
   }
 
   // Append the sets [a, b) of the held launch (a = held_done_) on every rank.
@@ -292,7 +309,7 @@ class RoundSampler {
       // kept fraction so far (first launch: 1/4), 5% + 64 ids of slack
       const double q = consumed_ ? std::max(1e-6, (double)std::max<uint64_t>(kept_, 1) / (double)consumed_) : 0.25;
       const double want = std::ceil((double)need / q * 1.05) + 64.0;
-      const uint64_t count = (uint64_t)std::min(want, (double)(1ull << 29) * W());
+      const uint64_t count = (uint64_t)std::min(want, (double)max_launch_ids(ctx_) * W());
       if (next_id_ + count > (1ull << 62)) fail(EIM_E_INVAL, "sample ids exhausted (< 2^62)");
       uint64_t lo, hi;
       eim_shard_range(next_id_, count, ctx_->rank, W(), &lo, &hi);
@@ -423,11 +440,15 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
           st->ms_select -= ms_since(tg);
           greedy_launch(ctx, 1, n, R_sel, total_i, ctx->C_snap.as<uint32_t>(), k, true);
           greedy_launch(ctx, 0, n, R, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, true);
-          cov = greedy_collect(ctx, 1, k, S.data(), nullptr);
-          cov_pre = greedy_collect(ctx, 0, k, S_pre.data(), nullptr);
+          cov = greedy_collect(ctx, 1, k, S.data(), nullptr, &st->ms_select_kernel);
+          cov_pre = greedy_collect(ctx, 0, k, S_pre.data(), nullptr, &st->ms_select_kernel);
           have_pre = true;
+          st->select_launches += 2;
+          st->select_picks += 2ull * k;
         } else {
-          cov = greedy(ctx, n, R, k, S.data(), nullptr);
+          cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
+          st->select_launches += 1;
+          st->select_picks += k;
         }
         st->ms_select += ms_since(ts);
       }
@@ -443,7 +464,10 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
       }
     }
     st->lb = LB;
-    const uint64_t theta = (uint64_t)std::ceil(p.lambda_s / LB);
+    const double theta_d = std::ceil(p.lambda_s / LB);
+    // set ids of the greedy's inverted index are 32-bit
+    if (!(theta_d < 4294967295.0)) fail(EIM_E_INVAL, "theta = ceil(lambda*/LB) exceeds 2^32 - 1 sets");
+    const uint64_t theta = (uint64_t)theta_d;
     if (have_pre) {
       // the loop stopped at round i with the sets of round i+1 appended: keep
       // max(theta, |R_i|) of them (the sequential loop's final |R|; with a
@@ -477,7 +501,9 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   }
   if (R != R_selected) {  // NodeSelection is deterministic: reuse the last run on the same R
     const auto ts = clk::now();
-    cov = greedy(ctx, n, R, k, S.data(), nullptr);
+    cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
+    st->select_launches += 1;
+    st->select_picks += k;
     st->ms_select += ms_since(ts);
   }
   std::memcpy(seeds_out, S.data(), (size_t)k * sizeof(uint32_t));

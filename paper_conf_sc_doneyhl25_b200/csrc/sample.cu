@@ -1028,17 +1028,24 @@ __global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* _
   if (edges_acc) atomicAdd(&ctl->edges, edges_acc);
 }
 
+// The walk store is a cache next to the graph store (not counted in
+// eim_graph_bytes); if it does not fit in device memory the walks run on the
+// plain store (lt_kernel), with the same results.
 static const uint4* lt_aug(eim_ctx* ctx, const eim_graph* gc, cudaStream_t st) {
-  if (std::getenv("EIM_NO_LT_AUG") || gc->packed || gc->weighted) return nullptr;
+  if (std::getenv("EIM_NO_LT_AUG") || gc->packed || gc->weighted || gc->aug_failed) return nullptr;
   eim_graph* g = const_cast<eim_graph*>(gc);  // lazily built cache of the (immutable) store
   if (!g->d_aug) {
     const uint64_t bytes = std::max<uint64_t>(g->view.m, 1) * sizeof(uint4);
-    EIM_CUDA(cudaMallocAsync(&g->d_aug, bytes, st));
+    if (cudaMallocAsync(&g->d_aug, bytes, st) != cudaSuccess) {
+      cudaGetLastError();
+      g->d_aug = nullptr;
+      g->aug_failed = true;
+      return nullptr;
+    }
     lt_aug_build_kernel<<<grid_for(ctx, g->view.m, 256), 256, 0, st>>>(g->view, static_cast<uint4*>(g->d_aug));
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
     g->aug_bytes = bytes;
-    g->bytes += bytes;
   }
   return static_cast<const uint4*>(g->d_aug);
 }
@@ -1627,12 +1634,33 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   return res;
 }
 
+uint64_t max_launch_ids(const eim_ctx* ctx) {
+  const uint32_t forced = env_u32("EIM_MAX_LAUNCH_IDS", 0);  // tests: force several launches per range
+  if (forced) return forced;
+  // the membership table of a launch holds >= 4 slots per expected member;
+  // keep it within 2^30 slots (8 GiB; the task pool adds 2 GiB)
+  const double mean = ctx->est_mean_size > 0 ? ctx->est_mean_size : 64.0;
+  const double cap = std::floor((double)(1ull << 30) / (4.0 * mean));
+  return (uint64_t)std::max(65536.0, std::min(cap, (double)(1ull << 29)));
+}
+
 SampleResult sample_range(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t seed,
                           uint64_t first, uint64_t count, uint64_t set_base, bool hist, uint32_t rflags) {
-  if (count == 0) return SampleResult{};
+  SampleResult tot;
   Round& rd = ctx->rounds[0];
-  round_launch(ctx, g, model, seed, first, count, set_base, hist, rd, ctx->stream, false, rflags);
-  return round_finalize(ctx, g, rd, count);
+  for (uint64_t done = 0; done < count;) {  // launches sized for the table budget
+    const uint64_t c = std::min(count - done, max_launch_ids(ctx));
+    round_launch(ctx, g, model, seed, first + done, c, set_base, hist, rd, ctx->stream, false, rflags);
+    const SampleResult r = round_finalize(ctx, g, rd, c);
+    tot.edges += r.edges;
+    tot.spilled += r.spilled;
+    tot.launches += r.launches;
+    tot.kernel_ms += r.kernel_ms;
+    tot.kept += r.kept;
+    tot.consumed += r.consumed;
+    done += c;
+  }
+  return tot;
 }
 
 }  // namespace eim

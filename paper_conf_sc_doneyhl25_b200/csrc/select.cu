@@ -320,7 +320,11 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
     a.dbg = ctx->stage_a.as<unsigned long long>();
   }
   void* args[] = {&a};
+  if (!S.ev[0])
+    for (cudaEvent_t& e : S.ev) EIM_CUDA(cudaEventCreate(&e));
+  EIM_CUDA(cudaEventRecord(S.ev[0], st));
   EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
+  EIM_CUDA(cudaEventRecord(S.ev[1], st));
   ctx->kernel_launches += 9;
   if (a.dbg) {
     std::vector<unsigned long long> hd((size_t)k * 3);
@@ -334,13 +338,19 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
   }
 }
 
-uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out) {
+uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
+                        double* kernel_ms) {
   GreedySlot& S = ctx->gs[slot];
   cudaStream_t st = S.stream;
   std::vector<unsigned long long> g(k);
   EIM_CUDA(cudaMemcpyAsync(seeds_out, S.seeds.p, (uint64_t)k * sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaMemcpyAsync(g.data(), S.gains.p, (uint64_t)k * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
+  if (kernel_ms) {
+    float ms = 0;
+    EIM_CUDA(cudaEventElapsedTime(&ms, S.ev[0], S.ev[1]));
+    *kernel_ms += ms;
+  }
   if (st != ctx->stream) {  // later work on the context's stream may reuse what the selection read
     EIM_CUDA(cudaEventRecord(ctx->ev1, st));
     EIM_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->ev1, 0));
@@ -354,9 +364,9 @@ uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out,
 }
 
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
-                uint64_t* gains_out) {
+                uint64_t* gains_out, double* kernel_ms) {
   greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, false);
-  return greedy_collect(ctx, 0, k, seeds_out, gains_out);
+  return greedy_collect(ctx, 0, k, seeds_out, gains_out, kernel_ms);
 }
 
 }  // namespace eim

@@ -148,6 +148,20 @@ def test_multirank_C3(eim):
         grp.close()
 
 
+def test_multirank_split_launches(eim, monkeypatch):
+    # several launches per range on every rank (table budget), plain and
+    # with source elimination; the launch sizes of all ranks must agree
+    monkeypatch.setenv("EIM_MAX_LAUNCH_IDS", "300")
+    off, nbr = inputs.config_graph("C1")
+    grp = Group(eim, 3, off, nbr)
+    try:
+        for model in ("IC", "LT"):
+            _check(eim, grp, off, nbr, 10, 0.3, 1.0, model, 4)
+            _check(eim, grp, off, nbr, 10, 0.3, 1.0, model, 4, flags=ELIM)
+    finally:
+        grp.close()
+
+
 def test_multirank_failure_releases_peers(eim):
     # one rank fails its argument check: the others must not wait for it
     off, nbr = inputs.config_graph("C1")

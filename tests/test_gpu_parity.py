@@ -620,3 +620,29 @@ def test_lt_walk_store_vs_row_offsets(eim, ctx, graphs, store, monkeypatch):
             _sets_equal(eim, ctx, g, off, nbr, "LT", 5, 2**40 + 7, 257)
         finally:
             eim.eim_graph_free(g)
+
+
+# Ranges above the membership-table budget are sampled in several launches
+# (ADVICE r1): forced tiny launches give the same sets and IMM results.
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_launches_split_by_table_budget(eim, ctx, graphs, model, monkeypatch):
+    off, nbr = graphs("C1")
+    g = eim.eim_load_graph_csr(ctx, off, nbr)
+    try:
+        monkeypatch.setenv("EIM_MAX_LAUNCH_IDS", "777")
+        _sets_equal(eim, ctx, g, off, nbr, model, 3, 5, 5000)
+        assert eim.eim_get_stats(ctx)["sample_launches"] >= 7
+        for flags in (0, ELIM, FRESH):
+            _imm_equal_flags(eim, ctx, g, off, nbr, 10, 0.3, 1.0, model, 2, flags)
+    finally:
+        eim.eim_graph_free(g)
+
+
+def test_select_seeds_rejects_duplicates(eim, ctx):
+    offs = np.array([0, 3, 5], dtype=np.uint64)
+    with pytest.raises(eim.EimError) as ei:
+        eim.eim_select_seeds(ctx, 10, offs, np.array([1, 2, 1, 4, 5], dtype=np.uint32), 2)
+    assert ei.value.status == eim.EIM_E_INVAL
+    # the same member in two different sets is fine
+    s, gn = eim.eim_select_seeds(ctx, 10, offs, np.array([1, 2, 3, 1, 5], dtype=np.uint32), 2)
+    assert s.tolist() == [1, 0] and gn.tolist() == [2, 0]  # all covered after the first pick: lowest id (R10)
