@@ -180,13 +180,18 @@ eim_status eim_load_graph_csr_ex(eim_ctx* ctx, uint32_t n, uint64_t m, const uin
  * graph loads but LT calls on it return EIM_E_INVAL.  The thresholds are
  * streamed from HBM (4 B per examined in-edge, one 16-B load per Philox
  * quad); LT keeps a per-edge cumulative array (+4 B per edge).
- * Errors: those of eim_load_graph_csr_ex; EIM_E_INVAL for EIM_G_LOG_ENCODE
- * together with edge_x. */
+ * With EIM_G_LOG_ENCODE the offsets and in-neighbours are log-encoded as
+ * for eim_load_graph_csr_ex while edge_x (and the LT cumulative
+ * weights) stay 32-bit; the results are those of the plain weighted store.
+ * Errors: those of eim_load_graph_csr_ex. */
 eim_status eim_load_graph_csr_weighted(eim_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* in_offsets,
                                        const uint32_t* in_neighbors, const uint32_t* edge_x, uint32_t gflags,
                                        eim_graph** out);
 /* Device bytes held by the graph store (plain: 8(n+1) + 4 max(m,4) + 4n;
- * log-encoded: the two container arrays incl. 2 padding words each).
+ * log-encoded: the two container arrays incl. 2 padding words each; with
+ * edge probabilities + 4 (m rounded up to 4, + 4) + 4 max(m,1) for x and
+ * the LT cumulative weights).  The LT walk store (a cache built on the
+ * first LT run of a plain graph) is not included.
  * Errors: EIM_E_STATE (freed graph), EIM_E_INVAL (bytes NULL). */
 eim_status eim_graph_bytes(const eim_graph* g, uint64_t* bytes);
 

@@ -50,7 +50,7 @@ void DevBuf::release() {
 
 void GreedySlot::release() {
   DevBuf* b[] = {&C_work, &inv_off, &inv_fill, &inv, &best, &seeds, &gains, &cand, &cidx, &arena_c, &selected, &covered,
-                 &scratch};
+                 &scratch, &dirty};
   for (DevBuf* x : b) x->release();
   for (cudaEvent_t& e : ev) {
     if (e) cudaEventDestroy(e);
@@ -261,7 +261,6 @@ eim_status eim_load_graph_csr_weighted(eim_ctx* ctx, uint32_t n, uint64_t m, con
   return guarded(ctx, [&] {
     if (!out) fail(EIM_E_INVAL, "out is NULL");
     if (gflags & ~(uint32_t)EIM_G_LOG_ENCODE) fail(EIM_E_INVAL, "unknown graph flag");
-    if (edge_x && (gflags & EIM_G_LOG_ENCODE)) fail(EIM_E_INVAL, "EIM_G_LOG_ENCODE with edge probabilities is not supported");
     *out = nullptr;
     if (n < 2 || n >= 0xFFFFFFFFu) fail(EIM_E_INVAL, "n must be in [2, 2^32-1)");
     if (m >= (1ull << 40)) fail(EIM_E_INVAL, "m must be < 2^40");
@@ -285,8 +284,8 @@ eim_status eim_load_graph_csr_weighted(eim_ctx* ctx, uint32_t n, uint64_t m, con
       graph_validate_and_thresholds(ctx, g);
       g->bytes = ((uint64_t)n + 1) * sizeof(uint64_t) + std::max<uint64_t>(m, 4) * sizeof(uint32_t) +
                  (uint64_t)n * sizeof(uint32_t);
+      if (edge_x) graph_attach_weights(ctx, g, edge_x);  // (its LT scan reads the plain offsets)
       if (gflags & EIM_G_LOG_ENCODE) graph_log_encode(ctx, g);
-      if (edge_x) graph_attach_weights(ctx, g, edge_x);
     } catch (...) {
       if (g->d_off) cudaFreeAsync(g->d_off, st);
       if (g->d_nbr) cudaFreeAsync(g->d_nbr, st);

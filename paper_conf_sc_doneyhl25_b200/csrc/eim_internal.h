@@ -66,6 +66,18 @@ struct WeightedGraphView {
   const uint32_t* cum;  // m: LT inclusive cumulative weights - 1 (valid when the graph's lt_ok)
 };
 
+// Log-encoded reverse CSR with general edge probabilities (NEXT-2 x NEXT-3):
+// offsets and in-neighbours packed as in PackedGraphView ("applied to
+// both the network data and the RRR sets"); the per-edge probabilities x
+// and LT cumulative weights cum stay 32-bit (they are not small integers).
+struct PackedWeightedGraphView {
+  uint32_t n;
+  uint64_t m;
+  PackedGraphView p;
+  const uint32_t* x;
+  const uint32_t* cum;
+};
+
 // Per-launch control block (device memory).  The counters that every group
 // polls or bumps sit on separate 128-byte lines.
 struct SampleCtl {
@@ -79,7 +91,8 @@ struct SampleCtl {
   unsigned long long tasks_pushed;              // tasks split off
   unsigned long long t_first, t_last_id, t_end;  // %globaltimer: first id taken, last id taken, last group exit (timeline)
   unsigned long long consumed;                   // source elimination: ids up to the last kept set
-  unsigned long long pad4[8];
+  unsigned long long ntickets;                   // IC: ids that need a traversal (the root pre-pass list)
+  unsigned long long pad4[7];
 };
 
 // Communicator of a multi-rank context (comm.cpp): NCCL across processes,
@@ -122,6 +135,7 @@ struct Round {
   DevBuf roots, kidx, ksizes;                    // source elimination: roots, kept-set index, kept sizes
   DevBuf dbg;                                    // EIM_DEBUG_TIMELINE per-sample records
   DevBuf queue;                                  // IC task pool (u32 seeds) + descriptors (all-zero between rounds)
+  DevBuf list;                                   // IC: s_local of the ids whose root has in-edges (pre-pass)
   uint64_t first = 0, count = 0, set_base = 0, seed = 0, pcap = 0, tcap = 0;
   bool qdirty = true;                            // descriptors need a memset before use
   uint32_t bits = 0;
@@ -142,7 +156,7 @@ struct Round {
 // Buffers and stream of one greedy NodeSelection (select.cu).  Two slots let
 // the IMM driver run the selections of two rounds concurrently.
 struct GreedySlot {
-  DevBuf C_work, inv_off, inv_fill, inv, best, seeds, gains, cand, cidx, arena_c, selected, covered, scratch;
+  DevBuf C_work, inv_off, inv_fill, inv, best, seeds, gains, cand, cidx, arena_c, selected, covered, scratch, dirty;
   cudaStream_t stream = nullptr;  // slot 0: the context's stream; slot 1: its own
   bool own_stream = false;
   cudaEvent_t ev[2] = {};          // around the pick kernel
@@ -166,6 +180,7 @@ struct eim_graph {
   eim::WeightedGraphView wview{};
   void* d_x = nullptr;
   void* d_cum = nullptr;
+  eim::PackedWeightedGraphView pwview{};  // packed && weighted
   void* d_aug = nullptr;         // LT walk store of the plain graph, built on the first LT run (uint4 per in-edge)
   uint64_t aug_bytes = 0;
   bool aug_failed = false;       // the walk store did not fit: LT runs on the plain store
@@ -205,6 +220,16 @@ struct eim_ctx {
 };
 
 namespace eim {
+
+// Calls f with the device view of g's store (every kernel that walks the
+// reverse CSR is a template over the view).
+template <class F>
+auto with_graph_view(const eim_graph* g, F&& f) {
+  if (g->packed && g->weighted) return f(g->pwview);
+  if (g->packed) return f(g->pview);
+  if (g->weighted) return f(g->wview);
+  return f(g->view);
+}
 
 constexpr uint32_t CTX_MAGIC = 0xE1A0C7A7u;
 constexpr uint32_t GRAPH_MAGIC = 0xE1A06A7Fu;

@@ -176,6 +176,12 @@ void graph_log_encode(eim_ctx* ctx, eim_graph* g) {
   g->pview = PackedGraphView{n, m, static_cast<const uint32_t*>(g->d_offw), static_cast<const uint32_t*>(g->d_nbrw),
                              boff, bnbr};
   g->packed = true;
+  const uint64_t wbytes = g->weighted ? g->bytes - ((uint64_t)(n + 1) * sizeof(uint64_t) +
+                                                    std::max<uint64_t>(m, 4) * sizeof(uint32_t) + (uint64_t)n * sizeof(uint32_t))
+                                      : 0;
+  if (g->weighted)  // the probabilities stay 32-bit next to the packed offsets and neighbours
+    g->pwview = PackedWeightedGraphView{n, m, g->pview, static_cast<const uint32_t*>(g->d_x),
+                                        static_cast<const uint32_t*>(g->d_cum)};
   // the plain store is gone: only the packed view may be used from here on
   EIM_CUDA(cudaFreeAsync(g->d_off, st));
   EIM_CUDA(cudaFreeAsync(g->d_nbr, st));
@@ -184,7 +190,7 @@ void graph_log_encode(eim_ctx* ctx, eim_graph* g) {
   g->view.off = nullptr;
   g->view.nbr = nullptr;
   g->view.thr = nullptr;
-  g->bytes = (woff + wnbr) * sizeof(uint32_t);
+  g->bytes = (woff + wnbr) * sizeof(uint32_t) + wbytes;
   EIM_CUDA(cudaStreamSynchronize(st));
 }
 
@@ -196,9 +202,7 @@ bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g) {
     unsigned int* d = reinterpret_cast<unsigned int*>(ctx->scratch.p);
     EIM_CUDA(cudaMemsetAsync(d, 0, sizeof(unsigned int), st));
     const uint32_t grid = grid_for(ctx, (uint64_t)g->view.n * 32, 256);
-    if (g->packed) proper_edge_kernel<<<grid, 256, 0, st>>>(g->pview, g->view.n, d);
-    else if (g->weighted) proper_edge_kernel<<<grid, 256, 0, st>>>(g->wview, g->view.n, d);
-    else proper_edge_kernel<<<grid, 256, 0, st>>>(g->view, g->view.n, d);
+    with_graph_view(g, [&](const auto& gv) { proper_edge_kernel<<<grid, 256, 0, st>>>(gv, g->view.n, d); });
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches += 1;
     unsigned int* h = static_cast<unsigned int*>(ctx->h_pinned);

@@ -30,6 +30,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <type_traits>
 #include <vector>
 #include <cstdlib>
 #include <string>
@@ -167,6 +168,7 @@ struct RoundView {
   uint32_t nohoist;              // 1: never use the hoisted edge draws (tests exercise the general path)
   unsigned long long* qc;        // task queue q: head at qc[16 q], tail at qc[16 q + 1] (one 128-B line each)
   uint32_t prefetch;             // L2-prefetch in_nbr of parked live edges (EIM_NO_PREFETCH=1 turns it off)
+  const uint32_t* list;          // IC: ticket t -> s_local (the ids whose root has in-edges; root pre-pass)
 };
 
 // Split-off tasks go to TQ queues (descriptor segments of tcap / TQ each):
@@ -714,20 +716,27 @@ __device__ __forceinline__ uint32_t traverse(const GV& g, const RoundView& R, Sa
 // the heavy samples that bound the round), then a new sample id; idle while
 // work is outstanding elsewhere (a running traversal may still split); exit
 // when every id is taken and nothing is outstanding.
-__device__ __forceinline__ bool take_id(SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
+__device__ __forceinline__ bool take_id(const RoundView& R, SampleCtl* ctl, uint64_t count, uint32_t& s_local) {
   if (vload(&ctl->ticket) < count) {
     atomicAdd(&ctl->outstanding, 1ull);  // before the ticket: an observer never sees "all taken, none outstanding" early
     const unsigned long long t = atomicAdd(&ctl->ticket, 1ull);
     if (t == 0) ctl->t_first = gtimer();
     if (t == count - 1) ctl->t_last_id = gtimer();
     if (t < count) {
-      gc.s_local = (uint32_t)t;
-      gc.nb = 0;
+      s_local = R.list[t];
       return true;
     }
     atomicAdd(&ctl->outstanding, ~0ull);
   }
   return false;
+}
+
+__device__ __forceinline__ bool take_id(const RoundView& R, SampleCtl* ctl, uint64_t count, GroupCtl& gc) {
+  uint32_t s_local;
+  if (!take_id(R, ctl, count, s_local)) return false;
+  gc.s_local = s_local;
+  gc.nb = 0;
+  return true;
 }
 
 // probe_first: new ids before tasks (the tasks are the suspended heavy
@@ -736,7 +745,7 @@ __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, u
                                            bool probe_first) {
   const volatile unsigned int* cp = R.cancel;
   if (cp[0] || cp[1]) return ACT_EXIT;  // cancelled or paused
-  if (probe_first && take_id(ctl, count, gc)) return ACT_LOCAL;
+  if (probe_first && take_id(R, ctl, count, gc)) return ACT_LOCAL;
   const unsigned long long tq = R.tcap / TQ;
   const uint32_t home = home_queue();
   // hint (pushed vs claimed, all queues): scan the queues only when some
@@ -768,7 +777,7 @@ __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, u
       return ACT_TASK;
     }
   }
-  if (!probe_first && take_id(ctl, count, gc)) return ACT_LOCAL;
+  if (!probe_first && take_id(R, ctl, count, gc)) return ACT_LOCAL;
   if (vload(&ctl->arena_fail)) return ACT_EXIT;  // the host redoes the round
   if (vload(&ctl->outstanding) == 0ull) {
     atomicMax(&ctl->t_end, gtimer());
@@ -795,6 +804,7 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV 
   const int gi = threadIdx.x / G, gtid = threadIdx.x % G, lane = threadIdx.x & 31;
   const SG<G> me = sg_at<G>(smem_raw, gi, W);
   GroupCtl& gc = *me.gc;
+  count = vload(&ctl->ntickets);  // the ids the root pre-pass left for a traversal
   if (gtid == 0) {
     gc.job.claim = 0;
     gc.job.open = 0;
@@ -845,6 +855,37 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV 
 template <int G, int NSG>
 size_t ic_smem(uint32_t W) {
   return NSG * sg_bytes<G>(W);
+}
+
+// Root pre-pass of an IC launch (Alg. 2 l.6): a thread per sample id draws
+// the root; a root without in-edges is the whole set (Alg. 2 l.10-20 examine
+// nothing), so its membership is recorded here, and every other id is
+// listed for ic_kernel's tickets.  On R-MAT most roots have no in-edges
+// (C2: 55 %): their samples no longer cost a group's decide/traverse round
+// trips and barriers.
+template <class GV>
+__global__ void ic_prepass_kernel(GV g, RoundView R, uint64_t count, SampleCtl* ctl, uint32_t* list, bool all) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i0 = (uint64_t)blockIdx.x * blockDim.x; i0 < count; i0 += stride) {
+    const uint64_t i = i0 + threadIdx.x;
+    bool trav = false;
+    if (i < count) {
+      const uint32_t root = all ? 0u : draw_root(R.base + i, g.n, R.K);
+      if (!all && g_off(g, (uint64_t)root + 1) == g_off(g, root)) {
+        if (table_insert(R.keys, R.bits, table_key((uint32_t)i, root)) < 0) mark_fail(ctl);
+        R.sizes[i] = 1;
+      } else {
+        trav = true;
+      }
+    }
+    // warp-aggregated append to the ticket list
+    const unsigned m = __ballot_sync(FULL, trav);
+    unsigned long long base = 0;
+    if (lane == 0 && m) base = atomicAdd(&ctl->ntickets, (unsigned long long)__popc(m));
+    base = __shfl_sync(FULL, base, 0);
+    if (trav) list[base + __popc(m & ((1u << lane) - 1u))] = (uint32_t)i;
+  }
 }
 
 // ---------------------------------------------------------------- LT
@@ -1213,7 +1254,7 @@ void ensure_sets(eim_ctx* ctx, uint64_t num_sets) {
 }
 
 void round_release(Round& rd) {
-  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.edges, &rd.fill, &rd.excl, &rd.ctl, &rd.queue, &rd.dbg,
+  DevBuf* b[] = {&rd.table, &rd.sizes, &rd.edges, &rd.fill, &rd.excl, &rd.ctl, &rd.queue, &rd.dbg, &rd.list,
                  &rd.roots, &rd.kidx, &rd.ksizes};
   for (DevBuf* x : b) x->release();
   for (cudaEvent_t& e : rd.ev) {
@@ -1267,10 +1308,10 @@ static void launch_ic(eim_ctx* ctx, const eim_graph* g, const RoundView& R, uint
                       cudaStream_t st, bool spare_sm_slot) {
   const uint32_t W = ring_w();
   const size_t smem = ic_smem<G, NSG>(W);
-  if (g->packed) launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, PackedGraphView>, g->pview, R, count, ctl, st, spare_sm_slot, W, smem);
-  else if (g->weighted)
-    launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, WeightedGraphView>, g->wview, R, count, ctl, st, spare_sm_slot, W, smem);
-  else launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, GraphView>, g->view, R, count, ctl, st, spare_sm_slot, W, smem);
+  with_graph_view(g, [&](const auto& gv) {
+    using GV = std::decay_t<decltype(gv)>;
+    launch_ic_on<G, NSG>(ctx, ic_kernel<G, NSG, GV>, gv, R, count, ctl, st, spare_sm_slot, W, smem);
+  });
 }
 
 
@@ -1296,7 +1337,8 @@ static RoundView round_view(Round& rd) {
                    philox_key(rd.seed),
                    std::getenv("EIM_NO_HOIST") ? 1u : 0u,
                    round_queues(rd),
-                   std::getenv("EIM_NO_PREFETCH") ? 0u : 1u};
+                   std::getenv("EIM_NO_PREFETCH") ? 0u : 1u,
+                   rd.list.as<uint32_t>()};
 }
 
 // one sampler launch over rd's remaining work, bracketed by events
@@ -1315,9 +1357,7 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
     uint64_t blocks = std::min<uint64_t>((uint64_t)std::max(1, per_sm) * ctx->sm_count, (rd.count + 255) / 256);
     const uint32_t grid = (uint32_t)std::max<uint64_t>(blocks, 1);
     if (aug) lt_aug_kernel<<<grid, 256, 0, st>>>(g->view, aug, R, rd.count, ctl);
-    else if (g->packed) lt_kernel<<<grid, 256, 0, st>>>(g->pview, R, rd.count, ctl);
-    else if (g->weighted) lt_kernel<<<grid, 256, 0, st>>>(g->wview, R, rd.count, ctl);
-    else lt_kernel<<<grid, 256, 0, st>>>(g->view, R, rd.count, ctl);
+    else with_graph_view(g, [&](const auto& gv) { lt_kernel<<<grid, 256, 0, st>>>(gv, R, rd.count, ctl); });
     EIM_CUDA(cudaGetLastError());
     ctx->kernel_launches++;
   }
@@ -1363,6 +1403,18 @@ static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_
   rd.nlaunch = 0;
   rd.waited = false;
   rd.elim_ready = false;
+  if (rd.model == EIM_IC) {
+    rd.list.reserve(count * sizeof(uint32_t), false, st);
+    const RoundView R = round_view(rd);
+    with_graph_view(g, [&](const auto& gv) {
+      // EIM_NO_PREPASS=1: every id gets a traversal (the singleton path is off)
+      ic_prepass_kernel<<<grid_for(ctx, count, 256), 256, 0, st>>>(gv, R, count, rd.ctl.as<SampleCtl>(),
+                                                                    rd.list.as<uint32_t>(),
+                                                                    std::getenv("EIM_NO_PREPASS") != nullptr);
+    });
+    EIM_CUDA(cudaGetLastError());
+    ctx->kernel_launches++;
+  }
   round_kernel(ctx, g, rd, st, spare_sm_slot);
 }
 
@@ -1440,7 +1492,8 @@ static void round_wait(eim_ctx* ctx, const eim_graph* g, Round& rd) {
       EIM_CUDA(cudaStreamWaitEvent(st, rd.ev[2 * rd.nlaunch - 1], 0));
       EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
       EIM_CUDA(cudaStreamSynchronize(st));
-      if ((h->ticket >= rd.count && h->outstanding == 0) || h->arena_fail) break;
+      const uint64_t ntk = rd.model == EIM_IC ? h->ntickets : rd.count;
+      if ((h->ticket >= ntk && h->outstanding == 0) || h->arena_fail) break;
       round_resume(ctx, g, rd, st);
     }
     rd.pend.kernel_ms += elapsed(counted);
@@ -1621,9 +1674,7 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
         (uint32_t)from, (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
         rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_sum, roots, kidx);
   };
-  if (g->packed) scatter(g->pview);
-  else if (g->weighted) scatter(g->wview);
-  else scatter(g->view);
+  with_graph_view(g, scatter);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;
   ctx->arena_used = cursor + total;

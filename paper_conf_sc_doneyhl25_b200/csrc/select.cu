@@ -137,7 +137,21 @@ struct GreedyArgs {
   uint32_t* seeds;
   unsigned long long* gains;
   unsigned long long* dbg;      // development: per-pick timestamps (nullable)
+  // chunked argmax (nc >= chunk_min): chunk_key[c] = the maximum key of
+  // chunk c's candidates, refreshed only for the chunks whose counts a
+  // cover touched (dirty[c]); the argmax then reads one key per chunk
+  unsigned long long* chunk_key;
+  uint8_t* dirty;
+  uint32_t chunk_min;
+  uint32_t chunk_shift;         // log2(candidates per chunk)
 };
+
+constexpr uint32_t CHUNK_SHIFT = 11;             // 2048 candidates (8 KB of counts) per chunk
+// opt-in (EIM_GREEDY_CHUNK_MIN): measured slower than the full scan at every
+// config (select per IMM: C2 2.07 -> 2.52 ms, C3 1.35 -> 1.97, C4 7.8 ->
+// 8.9, C5 73.5 -> 127 ms): the covers touch most chunks of the hub-heavy
+// counts, and marking them costs a store per decrement
+constexpr uint32_t CHUNK_MIN_DEFAULT = 0xFFFFFFFFu;
 
 __device__ __forceinline__ unsigned long long gtimer_ns() {
   unsigned long long t;
@@ -151,15 +165,55 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   __shared__ uint32_t big[BIG_CAP];
   __shared__ uint32_t nbig;
   if (threadIdx.x == 0) nbig = 0;
-  const uint32_t nc4 = ((*a.nc + 3u) & ~3u) / 4;
+  const uint32_t nc = *a.nc;
+  const uint32_t nc4 = ((nc + 3u) & ~3u) / 4;
   const uint4* W4 = reinterpret_cast<const uint4*>(a.W);
   const int lane = threadIdx.x & 31;
   const uint64_t warp = ((uint64_t)blockIdx.x * GB + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * GB) >> 5;
+  // ---- chunked argmax: for many candidates the full scan of W per pick
+  // (4 B per candidate from L2/HBM) is replaced by one key per chunk of
+  // 2^chunk_shift candidates; a cover marks the chunks whose counts it
+  // decrements, and only those are rescanned (by the block that owns them)
+  // before the next argmax.  The keys are exact whenever they are read, so
+  // the winner and the tie rule are the full scan's.
+  const bool chunked = nc >= a.chunk_min;
+  const uint32_t c4 = (1u << a.chunk_shift) / 4;  // uint4 per chunk (>= 1)
+  const uint32_t nchunks = (nc4 + c4 - 1) / c4;
+  const uint32_t cpb = (nchunks + gridDim.x - 1) / gridDim.x;  // chunks per block
+  const uint32_t cb0 = min(blockIdx.x * cpb, nchunks), cb1 = min(cb0 + cpb, nchunks);
   for (uint32_t j = 0; j < a.k; ++j) {
     if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j] = gtimer_ns();
-    // ---- argmax over this block's slice
     unsigned long long km = 0;
+    if (chunked) {
+      // refresh this block's dirty chunks (a warp per chunk), then reduce
+      // its chunk keys
+      for (uint32_t c = cb0 + (threadIdx.x >> 5); c < cb1; c += GB / 32) {
+        if (!__ldcg(a.dirty + c)) continue;
+        unsigned long long e = 0;
+        for (uint32_t i = c * c4 + lane; i < min((c + 1) * c4, nc4); i += 32) {
+          const uint4 w = __ldcg(W4 + i);
+          const uint32_t x = 4u * i;
+          e = umax64(e, umax64(umax64(ckey(w.x, x), ckey(w.y, x + 1)), umax64(ckey(w.z, x + 2), ckey(w.w, x + 3))));
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) e = umax64(e, __shfl_xor_sync(FULL, e, o));
+        if (lane == 0) {
+          a.chunk_key[c] = e;
+          a.dirty[c] = 0;
+        }
+      }
+      __syncthreads();
+      for (uint32_t c = cb0 + threadIdx.x; c < cb1; c += GB) km = umax64(km, a.chunk_key[c]);
+      km = block_max(km, red);
+      if (threadIdx.x == 0) a.blockmax[blockIdx.x] = km;
+      grid.sync();
+      if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 1] = gtimer_ns();
+      km = 0;
+      for (uint32_t b = threadIdx.x; b < gridDim.x; b += GB) km = umax64(km, a.blockmax[b]);
+      km = block_max(km, red);
+    } else {
+    // ---- argmax over this block's slice
     for (uint32_t i = blockIdx.x * GB + threadIdx.x; i < nc4; i += gridDim.x * GB) {
       const uint4 c = W4[i];
       const uint32_t x = 4u * i;
@@ -175,6 +229,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
     km = 0;
     for (uint32_t b = threadIdx.x; b < gridDim.x; b += GB) km = umax64(km, a.blockmax[b]);
     km = block_max(km, red);
+    }
     if (km == 0ull) {
       // every set is covered: the lowest unselected vertex id, gain 0
       if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -216,7 +271,11 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         }
         if (__shfl_sync(FULL, queued, 0)) continue;
 #pragma unroll 4
-        for (uint32_t t = lane; t < L; t += 32) atomicSub(&a.W[a.arena_c[st + t]], 1u);
+        for (uint32_t t = lane; t < L; t += 32) {
+          const uint32_t x = a.arena_c[st + t];
+          atomicSub(&a.W[x], 1u);
+          if (chunked) a.dirty[x >> a.chunk_shift] = 1;
+        }
       }
       __syncthreads();
       const uint32_t nb = min(nbig, BIG_CAP);
@@ -225,7 +284,11 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         const uint64_t st = a.set_start[i];
         const uint32_t L = a.set_len[i];
 #pragma unroll 4
-        for (uint32_t t = threadIdx.x; t < L; t += GB) atomicSub(&a.W[a.arena_c[st + t]], 1u);
+        for (uint32_t t = threadIdx.x; t < L; t += GB) {
+          const uint32_t x = a.arena_c[st + t];
+          atomicSub(&a.W[x], 1u);
+          if (chunked) a.dirty[x >> a.chunk_shift] = 1;
+        }
       }
       __syncthreads();
       if (threadIdx.x == 0) nbig = 0;
@@ -294,7 +357,15 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
   // two 148-block grids launched together take 2.0 ms (they do not overlap)
   if (concurrent) blocks = std::max(1u, blocks / 2);
   blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
-  S.best.reserve((uint64_t)blocks * sizeof(unsigned long long) + 64, false, st);
+  // chunked argmax from this many candidates on (EIM_GREEDY_CHUNK_MIN; 0:
+  // always) with 2^shift candidates per chunk (EIM_GREEDY_CHUNK_SHIFT, >= 2)
+  const char* cm = getenv("EIM_GREEDY_CHUNK_MIN");
+  const char* cs = getenv("EIM_GREEDY_CHUNK_SHIFT");
+  const uint32_t chunk_shift = std::max<uint32_t>(2, cs ? (uint32_t)strtoul(cs, nullptr, 10) : CHUNK_SHIFT);
+  const uint64_t nchunks_max = ((uint64_t)n >> chunk_shift) + 2;
+  S.best.reserve(((uint64_t)blocks + nchunks_max + 8) * sizeof(unsigned long long) + 64, false, st);
+  S.dirty.reserve(nchunks_max, false, st);
+  EIM_CUDA(cudaMemsetAsync(S.dirty.p, 1, nchunks_max, st));  // every chunk key is computed at the first pick
   uint32_t* zc = reinterpret_cast<uint32_t*>(S.best.as<unsigned long long>() + blocks);
   EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
   GreedyArgs a;
@@ -313,6 +384,10 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
   a.zc = zc;
   a.seeds = S.seeds.as<uint32_t>();
   a.gains = S.gains.as<unsigned long long>();
+  a.chunk_key = S.best.as<unsigned long long>() + blocks + 8;
+  a.dirty = S.dirty.as<uint8_t>();
+  a.chunk_min = cm ? (uint32_t)strtoul(cm, nullptr, 10) : CHUNK_MIN_DEFAULT;
+  a.chunk_shift = chunk_shift;
   a.dbg = nullptr;
   const char* gdbg = getenv("EIM_DEBUG_GREEDY");
   if (gdbg && slot == 0) {

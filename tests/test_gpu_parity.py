@@ -83,7 +83,9 @@ SPILL_MODES = {"default": {}, "spill_all": {"EIM_SPILL_QUADS": "1", "EIM_TASK_QU
                "nohoist": {"EIM_NO_HOIST": "1"},
                # probe-first rounds: nearly every root traversal is suspended into tasks;
                # and the id-order policy without probing
-               "probe": {"EIM_PROBE_QUADS": "2"}, "noprobe": {"EIM_PROBE_QUADS": "0"}}
+               "probe": {"EIM_PROBE_QUADS": "2"}, "noprobe": {"EIM_PROBE_QUADS": "0", "EIM_NO_PREPASS": "1"},
+               # the chunked argmax of the greedy for every candidate count, 8 per chunk
+               "chunked": {"EIM_GREEDY_CHUNK_MIN": "0", "EIM_GREEDY_CHUNK_SHIFT": "3"}}
 
 
 @pytest.fixture(params=list(SPILL_MODES))
@@ -128,7 +130,11 @@ def test_sample_rrr_special_graphs(eim, ctx, model, shape, spill_mode):
         eim.eim_graph_free(g)
 
 
-def test_select_seeds_on_oracle_arenas(eim, ctx, graphs):
+@pytest.mark.parametrize("chunked", ["-", "2", "5"])
+def test_select_seeds_on_oracle_arenas(eim, ctx, graphs, chunked, monkeypatch):
+    if chunked != "-":  # chunked argmax with 4 / 32 candidates per chunk
+        monkeypatch.setenv("EIM_GREEDY_CHUNK_MIN", "0")
+        monkeypatch.setenv("EIM_GREEDY_CHUNK_SHIFT", chunked)
     rng = np.random.default_rng(0)
     for trial in range(30):
         n = int(rng.integers(2, 300))
@@ -255,12 +261,15 @@ def test_C2_sets_exhaustive_coverage_and_imm(eim, ctx, graphs, monkeypatch):
         eim.eim_graph_free(g)
 
 
-def test_C3_sets_exhaustive_coverage_and_imm(eim, ctx, graphs):
+def test_C3_sets_exhaustive_coverage_and_imm(eim, ctx, graphs, monkeypatch):
     c = inputs.CONFIGS["C3"]
     off, nbr = graphs("C3")
     n = off.size - 1
     g = eim.eim_load_graph_csr(ctx, off, nbr)
     try:
+        with monkeypatch.context() as mp:  # the chunked argmax on a full-size selection
+            mp.setenv("EIM_GREEDY_CHUNK_MIN", "0")
+            _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
         st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
         assert st["theta"] == 58277
         C_gpu = eim.eim_get_coverage(ctx, n)
@@ -569,8 +578,40 @@ def test_weighted_special_cases(eim, ctx):
         eim.eim_imm_run(ctx, g, 1, 0.5, 1.0, "IC", 1)
     finally:
         eim.eim_graph_free(g)
-    with pytest.raises(eim.EimError):
-        eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC, edge_x=np.zeros(2, dtype=np.uint32))
+    # the packed weighted store (NEXT-2 x NEXT-3) keeps the LT rejection
+    g = eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC, edge_x=np.array([2**31, 2**31 - 1], dtype=np.uint32))
+    try:
+        with pytest.raises(eim.EimError) as ei:
+            eim.eim_imm_run(ctx, g, 1, 0.5, 1.0, "LT", 1)
+        assert ei.value.status == eim.EIM_E_INVAL
+    finally:
+        eim.eim_graph_free(g)
+
+
+# NEXT-2 x NEXT-3: log-encoded offsets/neighbours with per-edge probabilities
+# ("applied to both the network data and the RRR sets").
+@pytest.mark.parametrize("model", ["IC", "LT"])
+def test_weighted_log_encoded(eim, ctx, graphs, model, spill_mode):
+    off, nbr = graphs("C1")
+    x = _random_x(off, model, 11)
+    if model == "IC":
+        x = (x >> np.uint32(4)).astype(np.uint32)
+    g = eim.eim_load_graph_csr(ctx, off, nbr, gflags=LOGENC, edge_x=x)
+    try:
+        m = nbr.size
+        assert eim.eim_graph_bytes(g) == _packed_bytes(off, nbr) + 4 * ((m + 3) // 4 * 4 + 4) + 4 * max(m, 1)
+        go, gm = eim.eim_sample_rrr(ctx, g, model, 2, 0, 6000)
+        ro, rm, rex = oracle.sample(off, nbr, model, 2, 0, 6000, nthreads=NT, x=x)
+        assert np.array_equal(go, ro) and np.array_equal(gm, rm)
+        assert eim.eim_get_stats(ctx)["edges_examined"] == rex
+        for flags in (0, ELIM | FRESH):
+            seeds, theta, spread, st = eim.eim_imm_run(ctx, g, 5, 0.5, 1.0, model, 2, flags=flags)
+            ref = oracle.imm(off, nbr, 5, 0.5, 1.0, model, 2, nthreads=NT, flags=flags, x=x)
+            assert np.array_equal(seeds, ref["seeds"]) and theta == ref["theta"] and spread == ref["spread"]
+            for key in ("theta_i", "cov_i", "edges_examined", "arena_elems", "ids_sampled"):
+                assert st[key] == ref[key], key
+    finally:
+        eim.eim_graph_free(g)
 
 
 @pytest.mark.parametrize("model", ["IC", "LT"])
