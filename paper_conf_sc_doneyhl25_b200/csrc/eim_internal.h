@@ -315,6 +315,10 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
 // at the same time (each gets half the SMs).
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
                    uint32_t k, bool concurrent);
+// greedy_launch in two halves, so two slots' setups can overlap before the
+// host reads their candidate counts
+void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C);
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, bool concurrent);
 uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
                         double* kernel_ms = nullptr);
 

@@ -438,8 +438,10 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
           const auto tg = clk::now();
           sampler.grow(R, next, 0);  // appends the held sets, no launch
           st->ms_select -= ms_since(tg);
-          greedy_launch(ctx, 1, n, R_sel, total_i, ctx->C_snap.as<uint32_t>(), k, true);
-          greedy_launch(ctx, 0, n, R, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, true);
+          greedy_setup(ctx, 1, n, R_sel, total_i, ctx->C_snap.as<uint32_t>());
+          greedy_setup(ctx, 0, n, R, arena_cursor(ctx), ctx->C_total.as<uint32_t>());
+          greedy_picks(ctx, 1, n, R_sel, k, true);
+          greedy_picks(ctx, 0, n, R, k, true);
           cov = greedy_collect(ctx, 1, k, S.data(), nullptr, &st->ms_select_kernel);
           cov_pre = greedy_collect(ctx, 0, k, S_pre.data(), nullptr, &st->ms_select_kernel);
           have_pre = true;

@@ -302,6 +302,12 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
 
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
                    uint32_t k, bool concurrent) {
+  greedy_setup(ctx, slot, n, num_sets, total, C);
+  greedy_picks(ctx, slot, n, num_sets, k, concurrent);
+}
+
+// steps 1-2: candidates, remapped arena, inverted index (enqueued on the slot's stream)
+void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C) {
   GreedySlot& S = ctx->gs[slot];
   cudaStream_t st = S.stream;
   if (st != ctx->stream) {  // the slot's stream starts after the work enqueued so far (sets, C)
@@ -340,6 +346,15 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
         reinterpret_cast<unsigned long long*>(inv_off), S.inv.as<uint32_t>());
     EIM_CUDA(cudaGetLastError());
   }
+  ctx->kernel_launches += 7;
+}
+
+// step 3: the k picks in one cooperative grid kernel
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, bool concurrent) {
+  GreedySlot& S = ctx->gs[slot];
+  cudaStream_t st = S.stream;
+  uint32_t* pos = S.inv_fill.as<uint32_t>();
+  uint64_t* inv_off = S.inv_off.as<uint64_t>();
   // ---- 3. the k picks in one cooperative kernel
   S.covered.reserve(std::max<uint64_t>(num_sets, 1), false, st);
   S.selected.reserve((uint64_t)n + 4, false, st);
@@ -400,7 +415,7 @@ void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64
   EIM_CUDA(cudaEventRecord(S.ev[0], st));
   EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
   EIM_CUDA(cudaEventRecord(S.ev[1], st));
-  ctx->kernel_launches += 9;
+  ctx->kernel_launches += 2;
   if (a.dbg) {
     std::vector<unsigned long long> hd((size_t)k * 3);
     EIM_CUDA(cudaMemcpyAsync(hd.data(), a.dbg, (size_t)k * 24, cudaMemcpyDeviceToHost, st));

@@ -130,11 +130,11 @@ def test_sample_rrr_special_graphs(eim, ctx, model, shape, spill_mode):
         eim.eim_graph_free(g)
 
 
-@pytest.mark.parametrize("chunked", ["-", "2", "5"])
-def test_select_seeds_on_oracle_arenas(eim, ctx, graphs, chunked, monkeypatch):
-    if chunked != "-":  # chunked argmax with 4 / 32 candidates per chunk
+@pytest.mark.parametrize("mode", ["-", "chunk2", "chunk5"])
+def test_select_seeds_on_oracle_arenas(eim, ctx, graphs, mode, monkeypatch):
+    if mode.startswith("chunk"):  # chunked argmax with 4 / 32 candidates per chunk
         monkeypatch.setenv("EIM_GREEDY_CHUNK_MIN", "0")
-        monkeypatch.setenv("EIM_GREEDY_CHUNK_SHIFT", chunked)
+        monkeypatch.setenv("EIM_GREEDY_CHUNK_SHIFT", mode[5:])
     rng = np.random.default_rng(0)
     for trial in range(30):
         n = int(rng.integers(2, 300))
@@ -267,9 +267,11 @@ def test_C3_sets_exhaustive_coverage_and_imm(eim, ctx, graphs, monkeypatch):
     n = off.size - 1
     g = eim.eim_load_graph_csr(ctx, off, nbr)
     try:
-        with monkeypatch.context() as mp:  # the chunked argmax on a full-size selection
-            mp.setenv("EIM_GREEDY_CHUNK_MIN", "0")
-            _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
+        for env in ({"EIM_GREEDY_CHUNK_MIN": "0"},):  # the chunked argmax on a full-size selection
+            with monkeypatch.context() as mp:
+                for kk, vv in env.items():
+                    mp.setenv(kk, vv)
+                _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
         st = _imm_equal(eim, ctx, g, off, nbr, c["k"], c["eps"], c["ell"], "LT", 1)
         assert st["theta"] == 58277
         C_gpu = eim.eim_get_coverage(ctx, n)
