@@ -105,7 +105,7 @@ eim_status guarded(eim_ctx* ctx, F&& f) {
 bool ctx_ok(const eim_ctx* ctx) { return ctx && ctx->magic == CTX_MAGIC; }
 
 void free_ctx_buffers(eim_ctx* c) {
-  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->ctl, &c->C_total, &c->C_snap, &c->scratch,
+  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->ctl, &c->C_total, &c->C_snap, &c->edges_acc, &c->scratch,
                     &c->stage_a, &c->stage_b, &c->stage_c};
   for (DevBuf* b : bufs) b->release();
   for (GreedySlot& g : c->gs) g.release();
@@ -391,10 +391,11 @@ eim_status eim_sample_rrr_ex(eim_ctx* ctx, const eim_graph* g, eim_model model, 
     const uint64_t launches0 = ctx->kernel_launches;
     ctx->cov_n = 0;
     arena_reset(ctx, g->packed ? bit_width((uint64_t)g->view.n - 1) : 32u);
+    edges_reset(ctx);
     const SampleResult r = sample_range(ctx, g, model, seed, first_id, count, first_id, false,
                                         (flags & EIM_F_SOURCE_ELIM) ? RF_DROP_ROOT : 0u);
     std::memset(&ctx->last_stats, 0, sizeof(eim_stats));
-    ctx->last_stats.edges_examined = r.edges;
+    ctx->last_stats.edges_examined = edges_read(ctx);
     ctx->last_stats.spilled_samples = r.spilled;
     ctx->last_stats.sample_launches = r.launches;
     ctx->last_stats.ms_sample_kernel = r.kernel_ms;

@@ -122,7 +122,7 @@ struct LocalGroup;
 enum : uint32_t { RF_DROP_ROOT = 1u, RF_DROP_EMPTY = 2u };
 
 struct SampleResult {
-  uint64_t edges = 0;
+  uint64_t edges = 0;     // (unused: examined edges accumulate on the device, edges_read)
   uint64_t spilled = 0;   // samples finished in the shared frontier queue
   uint32_t launches = 0;
   double kernel_ms = 0;
@@ -210,6 +210,7 @@ struct eim_ctx {
   uint32_t arena_b = 32;                        // bits per arena element: 32 plain, else log-encoded (R24)
   // per-graph vectors
   eim::DevBuf C_total, C_snap;                  // coverage counts of R; snapshot for a concurrent selection
+  eim::DevBuf edges_acc;                        // examined edges / walk steps of the current call (u64)
   eim::GreedySlot gs[2];                        // greedy NodeSelection slots
   eim::DevBuf scratch;        // CUB temp storage
   eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
@@ -247,6 +248,10 @@ bool graph_has_proper_edge(eim_ctx* ctx, const eim_graph* g);
 // Sample ids per launch that keep the round's membership table within its
 // memory budget (from the mean set size of earlier launches).
 uint64_t max_launch_ids(const eim_ctx* ctx);
+// Examined in-edges (IC) / walk steps (LT) of the appended sets accumulate
+// in a device counter (no host round trip per launch): reset, read (syncs).
+void edges_reset(eim_ctx* ctx);
+uint64_t edges_read(eim_ctx* ctx);
 // Samples ids [first, first+count) into ctx->arena; set index = id - set_base
 // (in launches of at most max_launch_ids ids).
 // Histogram into C when hist is true.  (= round_launch + round_finalize)

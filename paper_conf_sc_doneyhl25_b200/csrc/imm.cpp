@@ -192,7 +192,6 @@ class RoundSampler {
  private:
   cudaStream_t stream_of(const Round& rd) const { return &rd == &ctx_->rounds[0] ? ctx_->rstream[0] : ctx_->rstream[1]; }
   void account(const SampleResult& r) {
-    st_->edges_examined += r.edges;
     st_->spilled_samples += r.spilled;
     st_->sample_launches += r.launches;
     st_->ms_sample_kernel += r.kernel_ms;
@@ -395,6 +394,8 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   // fresh arena + coverage for this graph; R is log-encoded with the graph (NEXT-2)
   const uint32_t arena_b = g->packed ? bit_width((uint64_t)n - 1) : 32u;
   arena_reset(ctx, arena_b);
+  edges_reset(ctx);
+  uint64_t dropped_edges = 0;  // examined edges of sets dropped again (paired rounds)
   ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
   EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
   RoundSampler sampler(ctx, g, model, seed, st, elim);
@@ -476,9 +477,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
       // fresh final phase the estimation phase sampled exactly |R_i|)
       const uint64_t keep = fresh ? R_selected : std::max<uint64_t>(theta, R_selected);
       if (keep < R) {
-        uint64_t dropped_edges = 0;
         drop_sets(ctx, g, model == EIM_IC, keep, R, &dropped_edges);
-        st->edges_examined -= dropped_edges;
         st->ids_sampled -= R - keep;
         R = keep;
       } else {
@@ -509,6 +508,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
     st->ms_select += ms_since(ts);
   }
   std::memcpy(seeds_out, S.data(), (size_t)k * sizeof(uint32_t));
+  st->edges_examined = edges_read(ctx) - dropped_edges;
   st->theta = R;
   st->cov = cov;
   st->arena_elems = arena_cursor(ctx);

@@ -1092,6 +1092,8 @@ static const uint4* lt_aug(eim_ctx* ctx, const eim_graph* gc, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- output
+__global__ void add_u64_kernel(unsigned long long* acc, const unsigned long long* x) { *acc += *x; }
+
 __global__ void sizes_to_offsets_kernel(const uint32_t* __restrict__ sizes, uint64_t count,
                                         uint64_t* __restrict__ out) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -1370,6 +1372,12 @@ static void round_kernel(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream
 // table + queue sizing, memsets and the first launch of rd's range on st
 static void round_start(eim_ctx* ctx, const eim_graph* g, Round& rd, cudaStream_t st, bool spare_sm_slot) {
   const uint64_t count = rd.count;
+  if (st != ctx->stream) {
+    // the round's buffers may still be read by the previous round's
+    // finalize (scatter) on the context's stream: start after it
+    EIM_CUDA(cudaEventRecord(ctx->ev0, ctx->stream));
+    EIM_CUDA(cudaStreamWaitEvent(st, ctx->ev0, 0));
+  }
   rd.table.reserve(8ull << rd.bits, false, st);
   EIM_CUDA(cudaMemsetAsync(rd.table.p, 0, 8ull << rd.bits, st));
   if (rd.model == EIM_IC) {
@@ -1648,15 +1656,20 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
   sizes_to_offsets_kernel<<<grid_for(ctx, nsets + 1, 256), 256, 0, st>>>(sizes, nsets, excl);
   EIM_CUDA(cudaGetLastError());
   const bool ic = rd.model == EIM_IC;
-  unsigned long long* d_edges_sum = &ctl->edges;  // IC: summed by the scatter; LT: reduced from per-walk steps
+  // examined edges go to the context's device accumulator (edges_read):
+  // IC summed by the scatter, LT reduced from the per-walk steps and added
+  unsigned long long* d_edges_acc = ctx->edges_acc.as<unsigned long long>();
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, excl, excl, nsets + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>() + from, d_edges_sum,
+  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(nullptr, tmp2, rd.edges.as<unsigned long long>() + from, &ctl->edges,
                                            consumed - from, st));
   ctx->scratch.reserve(std::max<size_t>(std::max(tmp, tmp2), 1 << 20), false, st);
   EIM_CUDA(cub::DeviceScan::ExclusiveSum(ctx->scratch.p, tmp, excl, excl, nsets + 1, st));
-  if (!ic) EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>() + from, d_edges_sum,
-                                           consumed - from, st));
-  else EIM_CUDA(cudaMemsetAsync(d_edges_sum, 0, sizeof(unsigned long long), st));
+  if (!ic) {
+    EIM_CUDA(cub::DeviceReduce::Sum(ctx->scratch.p, tmp2, rd.edges.as<unsigned long long>() + from, &ctl->edges,
+                                    consumed - from, st));
+    add_u64_kernel<<<1, 1, 0, st>>>(d_edges_acc, &ctl->edges);
+    EIM_CUDA(cudaGetLastError());
+  }
   EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + nsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
   EIM_CUDA(cudaStreamSynchronize(st));
   const uint64_t total = h->ticket, cursor = ctx->arena_used;
@@ -1672,17 +1685,26 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
         rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
         (uint32_t)from, (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
-        rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_sum, roots, kidx);
+        rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_acc, roots, kidx);
   };
   with_graph_view(g, scatter);
   EIM_CUDA(cudaGetLastError());
   ctx->kernel_launches += 6;
   ctx->arena_used = cursor + total;
-  EIM_CUDA(cudaMemcpyAsync(&h->edges, d_edges_sum, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
-  EIM_CUDA(cudaStreamSynchronize(st));
-  res.edges = h->edges;
   ctx->est_mean_size = std::max(1.0, (double)(total + (drop_root ? consumed : 0)) / (double)(consumed - from));
   return res;
+}
+
+void edges_reset(eim_ctx* ctx) {
+  ctx->edges_acc.reserve(64, false, ctx->stream);
+  EIM_CUDA(cudaMemsetAsync(ctx->edges_acc.p, 0, sizeof(unsigned long long), ctx->stream));
+}
+
+uint64_t edges_read(eim_ctx* ctx) {
+  uint64_t* h = reinterpret_cast<uint64_t*>(static_cast<char*>(ctx->h_pinned) + 3584);
+  EIM_CUDA(cudaMemcpyAsync(h, ctx->edges_acc.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  EIM_CUDA(cudaStreamSynchronize(ctx->stream));
+  return *h;
 }
 
 uint64_t max_launch_ids(const eim_ctx* ctx) {
