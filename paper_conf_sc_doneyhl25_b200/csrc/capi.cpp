@@ -105,7 +105,8 @@ eim_status guarded(eim_ctx* ctx, F&& f) {
 bool ctx_ok(const eim_ctx* ctx) { return ctx && ctx->magic == CTX_MAGIC; }
 
 void free_ctx_buffers(eim_ctx* c) {
-  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->ctl, &c->C_total, &c->C_snap, &c->edges_acc, &c->scratch,
+  DevBuf* bufs[] = {&c->arena, &c->set_start, &c->set_len, &c->ctl, &c->C_total, &c->C_snap, &c->C_snap2, &c->edges_acc,
+                    &c->scratch,
                     &c->stage_a, &c->stage_b, &c->stage_c};
   for (DevBuf* b : bufs) b->release();
   for (GreedySlot& g : c->gs) g.release();
@@ -157,8 +158,10 @@ eim_ctx* new_ctx(int device, int rank, int world, uint64_t stream, MakeComm&& ma
     EIM_CUDA(cudaStreamCreateWithFlags(&c->rstream[1], cudaStreamNonBlocking));
     EIM_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
     c->gs[0].stream = c->stream;
-    EIM_CUDA(cudaStreamCreateWithFlags(&c->gs[1].stream, cudaStreamNonBlocking));
-    c->gs[1].own_stream = true;
+    for (int q = 1; q < 3; ++q) {
+      EIM_CUDA(cudaStreamCreateWithFlags(&c->gs[q].stream, cudaStreamNonBlocking));
+      c->gs[q].own_stream = true;
+    }
     EIM_CUDA(cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device));
     // keep freed stream-ordered memory in the device's pool: reloading a
     // graph or regrowing a buffer reuses it instead of cudaMalloc/cudaFree

@@ -209,9 +209,9 @@ struct eim_ctx {
   uint64_t arena_used = 0;                      // arena elements in use (host is the authority)
   uint32_t arena_b = 32;                        // bits per arena element: 32 plain, else log-encoded (R24)
   // per-graph vectors
-  eim::DevBuf C_total, C_snap;                  // coverage counts of R; snapshot for a concurrent selection
+  eim::DevBuf C_total, C_snap, C_snap2;         // coverage counts of R; snapshots for concurrent selections
   eim::DevBuf edges_acc;                        // examined edges / walk steps of the current call (u64)
-  eim::GreedySlot gs[2];                        // greedy NodeSelection slots
+  eim::GreedySlot gs[3];                        // greedy NodeSelection slots
   eim::DevBuf scratch;        // CUB temp storage
   eim::DevBuf stage_a, stage_b, stage_c;  // export / exchange staging
   void* h_pinned = nullptr;   // small pinned host scratch
@@ -316,14 +316,15 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
                 uint64_t* gains_out, double* kernel_ms = nullptr);
 // The same, split: enqueue on slot `slot` (its stream waits for the context's
 // stream first), then wait and read the result.  C and the arena prefix must
-// stay unchanged until greedy_collect.  concurrent: another selection runs
-// at the same time (each gets half the SMs).
+// stay unchanged until greedy_collect.
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
-                   uint32_t k, bool concurrent);
+                   uint32_t k, uint32_t concurrent);
 // greedy_launch in two halves, so two slots' setups can overlap before the
 // host reads their candidate counts
 void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C);
-void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, bool concurrent);
+// concurrent: the number of selections running at the same time (each
+// gets that share of the SMs)
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t concurrent);
 uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
                         double* kernel_ms = nullptr);
 

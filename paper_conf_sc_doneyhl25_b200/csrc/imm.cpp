@@ -121,12 +121,11 @@ std::vector<uint64_t> allgather_host(eim_ctx* ctx, Exchange& ex, uint64_t v) {
 // part of each requested range [|R|, to); with W > 1 the parts are then
 // exchanged (exchange_sets), so every rank holds all sets in sample-id order.
 //
-// Lookahead (default on; EIM_NO_LOOKAHEAD=1 turns it off): when the next
-// estimation round adds no more ids than this one, or the IMM driver expects
-// it to be needed (next_likely), one launch samples both and the next
-// round's sets are appended from the same round table without a launch --
-// one round tail (the heavy samples' critical paths; for LT the longest
-// walk) instead of two.  Sample ids are fixed labels, so the sets are the
+// Lookahead (default on; EIM_NO_LOOKAHEAD=1 turns it off): the IMM driver
+// may ask one launch to sample the ids of later rounds too (extend_to); their
+// sets are then appended from the same round table without a launch -- one
+// round tail (the heavy samples' critical paths; for LT the longest walk)
+// instead of several.  Sample ids are fixed labels, so the sets are the
 // same; if the estimation loop stops first the extra sets are discarded.
 //
 // Speculation (opt-in EIM_SPECULATE=1, one GPU): the next round's ids are
@@ -161,19 +160,20 @@ class RoundSampler {
     ex_.mem_recv.release();
   }
 
-  // make sets [R, to) final; next_to: the next round's target (lookahead /
-  // speculation); next_likely: the next round is expected to be needed
-  void grow(uint64_t& R, uint64_t to, uint64_t next_to, bool next_likely = false) {
+  // make sets [R, to) final; extend_to > to: the launch also samples the
+  // later rounds' ids [to, extend_to) (lookahead), or the next round is
+  // launched speculatively (EIM_SPECULATE)
+  void grow(uint64_t& R, uint64_t to, uint64_t extend_to) {
     if (to <= R) return;
     const auto t0 = clk::now();
     if (elim_) {
       grow_elim(R, to);
     } else if (speculate_) {
       st_->ids_sampled += to - R;
-      grow_speculate(R, to, next_to);
+      grow_speculate(R, to, extend_to);
     } else {
       st_->ids_sampled += to - R;
-      grow_shared(R, to, next_to, next_likely);
+      grow_shared(R, to, extend_to);
     }
     st_->ms_sample += ms_since(t0);
   }
@@ -201,7 +201,7 @@ class RoundSampler {
   // ---- plain runs, any number of ranks.  The held launch covers set
   // indices [launch_first_, launch_end_) (this rank: [my_lo_, my_hi_));
   // sets [launch_first_, held_done_) are appended on every rank.
-  void grow_shared(uint64_t& R, uint64_t to, uint64_t next_to, bool next_likely) {
+  void grow_shared(uint64_t& R, uint64_t to, uint64_t extend_to) {
     if (held_) {
       if (held_done_ == R) {
         append_part(R, std::min(launch_end_, to));
@@ -220,7 +220,7 @@ class RoundSampler {
       append_part(R, R + cap);
       R += cap;
     }
-    uint64_t end = (lookahead_ && next_to > to && (next_to - to <= to - R || next_likely)) ? next_to : to;
+    uint64_t end = (lookahead_ && extend_to > to) ? extend_to : to;
     if (end - R > cap) end = to;
     launch_range(R, end);
     append_part(R, to);
@@ -399,55 +399,89 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   ctx->C_total.reserve((uint64_t)n * sizeof(uint32_t), false, s);
   EIM_CUDA(cudaMemsetAsync(ctx->C_total.p, 0, (uint64_t)n * sizeof(uint32_t), s));
   RoundSampler sampler(ctx, g, model, seed, st, elim);
-  std::vector<uint32_t> S(k), S_pre(k);
-  uint64_t R = 0, cov = 0, cov_pre = 0;
+  std::vector<uint32_t> S(k);
+  uint64_t R = 0, cov = 0;
   uint64_t R_selected = UINT64_MAX;  // |R| the last NodeSelection ran on
-  bool have_pre = false;             // S_pre / cov_pre: NodeSelection on the current R, run ahead
-  // Paired rounds: when one lookahead launch has sampled rounds i and i+1,
-  // both NodeSelections run concurrently (slots 0 and 1, on R_{i+1} and on
-  // R_i with a snapshot of its counts).  If round i's stop test breaks, the
-  // sets of round i+1 that the final phase does not need are dropped again
+  // Run-ahead selections: when one launch has sampled rounds i..J (J <= i+2),
+  // the NodeSelections of all of them run concurrently (greedy slots 0..J-i,
+  // each on its prefix R_t of the arena with a snapshot of C taken after
+  // round t's append), and the later rounds' results wait here.  If round t
+  // stops the loop, the sets the final phase does not need are dropped again
   // (drop_sets: counts, arena, examined edges), so every reported number is
   // the sequential loop's.  One GPU, plain 32-bit arena; EIM_NO_PAIR=1: off.
+  struct Pre {
+    uint64_t R, cov;
+    std::vector<uint32_t> S;
+  };
+  std::vector<Pre> pre;
   const bool pairing = ctx->world == 1 && !elim && g->view.off && !g->packed && std::getenv("EIM_NO_PAIR") == nullptr;
   double LB = 1.0;
   auto theta_round = [&](uint32_t i) { return (uint64_t)std::ceil(std::ldexp(p.lambda_p, (int)i) / (double)n); };
+  auto has_round = [&](uint32_t i) { return (double)i < p.log2n; };
+  // Round t is predicted not to stop the loop when the last round's coverage
+  // fraction f, times 2^t, stays below (1+eps') by a margin of three
+  // standard errors of f (the fraction falls slowly as R grows: C2 0.098,
+  // 0.094, 0.090, 0.087, 0.085).  A scheduling guess only: the results never
+  // depend on it (a wrong guess samples ids the loop does not use).
+  auto continues = [&](uint32_t t) {
+    if (R_selected == UINT64_MAX || R_selected == 0) return false;
+    const double f = (double)cov / (double)R_selected;
+    if (f <= 0.0) return true;
+    const double m = std::min(0.95, std::max(0.5, 1.0 - 3.0 * std::sqrt((1.0 - f) / (f * (double)R_selected))));
+    return f * std::ldexp(1.0, (int)t) < m * (1.0 + p.eps_p);
+  };
   try {
-    for (uint32_t i = 1; (double)i < p.log2n; ++i) {
-      const uint64_t next = (double)(i + 1) < p.log2n ? theta_round(i + 1) : 0;
+    for (uint32_t i = 1; has_round(i); ++i) {
       uint64_t R_sel = R;
-      if (have_pre) {  // this round's selection ran with the previous one
-        have_pre = false;
-        S.swap(S_pre);
-        cov = cov_pre;
+      if (!pre.empty()) {  // this round's selection ran with an earlier one
+        R_sel = pre.front().R;
+        cov = pre.front().cov;
+        S.swap(pre.front().S);
+        pre.erase(pre.begin());
       } else {
-        // round i is expected not to stop the loop when the coverage fraction
-        // of the previous round is below half of what round i needs (the
-        // fraction falls slowly as R grows: C2 0.098, 0.094, 0.090, 0.087,
-        // 0.085); then round i+1 will be needed and is sampled in the same
-        // launch.  A scheduling guess only: the results never depend on it.
-        const bool next_likely = R_selected != UINT64_MAX && R_selected > 0 &&
-                                 (double)cov / (double)R_selected * std::ldexp(1.0, (int)i) < 0.5 * (1.0 + p.eps_p);
-        sampler.grow(R, theta_round(i), next, next_likely);
+        // the launch extent: round i+1 when it adds no more ids than round i
+        // (cheap even if round i stops) or round i is predicted to continue;
+        // round i+2 as well when rounds i and i+1 are both predicted to
+        // continue (run-ahead selections only)
+        uint32_t J = i;
+        if (has_round(i + 1) && (theta_round(i + 1) - theta_round(i) <= theta_round(i) - R || continues(i))) {
+          J = i + 1;
+          if (pairing && has_round(i + 2) && continues(i) && continues(i + 1)) J = i + 2;
+        }
+        sampler.grow(R, theta_round(i), theta_round(J));
         R_sel = R;
         const auto ts = clk::now();
-        if (pairing && next > R && sampler.holds(R, next)) {
-          const uint64_t total_i = arena_cursor(ctx);
-          ctx->C_snap.reserve((uint64_t)n * sizeof(uint32_t), false, s);
-          EIM_CUDA(cudaMemcpyAsync(ctx->C_snap.p, ctx->C_total.p, (uint64_t)n * sizeof(uint32_t),
-                                   cudaMemcpyDeviceToDevice, s));
-          const auto tg = clk::now();
-          sampler.grow(R, next, 0);  // appends the held sets, no launch
-          st->ms_select -= ms_since(tg);
-          greedy_setup(ctx, 1, n, R_sel, total_i, ctx->C_snap.as<uint32_t>());
-          greedy_setup(ctx, 0, n, R, arena_cursor(ctx), ctx->C_total.as<uint32_t>());
-          greedy_picks(ctx, 1, n, R_sel, k, true);
-          greedy_picks(ctx, 0, n, R, k, true);
-          cov = greedy_collect(ctx, 1, k, S.data(), nullptr, &st->ms_select_kernel);
-          cov_pre = greedy_collect(ctx, 0, k, S_pre.data(), nullptr, &st->ms_select_kernel);
-          have_pre = true;
-          st->select_launches += 2;
-          st->select_picks += 2ull * k;
+        if (pairing && J > i && sampler.holds(R, theta_round(i + 1))) {
+          const uint32_t nsel = J - i + 1;
+          std::vector<uint64_t> Rs(nsel), totals(nsel);
+          DevBuf* snaps[2] = {&ctx->C_snap, &ctx->C_snap2};
+          for (uint32_t t = 0; t < nsel; ++t) {
+            Rs[t] = R;
+            totals[t] = arena_cursor(ctx);
+            if (t + 1 == nsel) break;
+            snaps[t]->reserve((uint64_t)n * sizeof(uint32_t), false, s);
+            EIM_CUDA(cudaMemcpyAsync(snaps[t]->p, ctx->C_total.p, (uint64_t)n * sizeof(uint32_t),
+                                     cudaMemcpyDeviceToDevice, s));
+            const auto tg = clk::now();
+            sampler.grow(R, theta_round(i + t + 1), theta_round(J));  // appends the held sets, no launch
+            st->ms_select -= ms_since(tg);
+          }
+          // slot nsel-1-t runs round i+t (round J, on the live counts, in slot 0)
+          for (uint32_t t = 0; t < nsel; ++t)
+            greedy_setup(ctx, nsel - 1 - t, n, Rs[t], totals[t],
+                         t + 1 == nsel ? ctx->C_total.as<uint32_t>() : snaps[t]->as<uint32_t>());
+          for (uint32_t t = 0; t < nsel; ++t) greedy_picks(ctx, nsel - 1 - t, n, Rs[t], k, nsel);
+          for (uint32_t t = 0; t < nsel; ++t) {
+            if (t == 0) {
+              cov = greedy_collect(ctx, nsel - 1, k, S.data(), nullptr, &st->ms_select_kernel);
+            } else {
+              Pre q{Rs[t], 0, std::vector<uint32_t>(k)};
+              q.cov = greedy_collect(ctx, nsel - 1 - t, k, q.S.data(), nullptr, &st->ms_select_kernel);
+              pre.push_back(std::move(q));
+            }
+          }
+          st->select_launches += nsel;
+          st->select_picks += (uint64_t)nsel * k;
         } else {
           cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
           st->select_launches += 1;
@@ -471,22 +505,24 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
     // set ids of the greedy's inverted index are 32-bit
     if (!(theta_d < 4294967295.0)) fail(EIM_E_INVAL, "theta = ceil(lambda*/LB) exceeds 2^32 - 1 sets");
     const uint64_t theta = (uint64_t)theta_d;
-    if (have_pre) {
-      // the loop stopped at round i with the sets of round i+1 appended: keep
-      // max(theta, |R_i|) of them (the sequential loop's final |R|; with a
-      // fresh final phase the estimation phase sampled exactly |R_i|)
+    if (R > R_selected && R_selected != UINT64_MAX) {
+      // the loop stopped at a round whose later rounds' sets are appended:
+      // keep max(theta, |R_i|) of them (the sequential loop's final |R|; with
+      // a fresh final phase the estimation phase sampled exactly |R_i|)
       const uint64_t keep = fresh ? R_selected : std::max<uint64_t>(theta, R_selected);
       if (keep < R) {
         drop_sets(ctx, g, model == EIM_IC, keep, R, &dropped_edges);
         st->ids_sampled -= R - keep;
         R = keep;
-      } else {
-        R_selected = R;  // the run-ahead selection is the one on R
-        S.swap(S_pre);
-        cov = cov_pre;
       }
-      have_pre = false;
+      for (Pre& q : pre)  // a run-ahead selection on exactly the final R is the final one
+        if (q.R == R) {
+          R_selected = R;
+          S.swap(q.S);
+          cov = q.cov;
+        }
     }
+    pre.clear();
     if (fresh) {  // R23: the final sets are drawn afresh from ids 2^61..
       sampler.restart(EIM_FRESH_BASE);
       arena_reset(ctx, arena_b);

@@ -301,7 +301,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
 }  // namespace
 
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
-                   uint32_t k, bool concurrent) {
+                   uint32_t k, uint32_t concurrent) {
   greedy_setup(ctx, slot, n, num_sets, total, C);
   greedy_picks(ctx, slot, n, num_sets, k, concurrent);
 }
@@ -350,7 +350,7 @@ void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_
 }
 
 // step 3: the k picks in one cooperative grid kernel
-void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, bool concurrent) {
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t concurrent) {
   GreedySlot& S = ctx->gs[slot];
   cudaStream_t st = S.stream;
   uint32_t* pos = S.inv_fill.as<uint32_t>();
@@ -370,7 +370,7 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   // selections of the paired rounds 1 and 2), 74 + 74 blocks take 1.33 ms
   // against 1.93 ms for the two one after the other on 148 blocks, while
   // two 148-block grids launched together take 2.0 ms (they do not overlap)
-  if (concurrent) blocks = std::max(1u, blocks / 2);
+  if (concurrent > 1) blocks = std::max(1u, blocks / concurrent);
   blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
   // chunked argmax from this many candidates on (EIM_GREEDY_CHUNK_MIN; 0:
   // always) with 2^shift candidates per chunk (EIM_GREEDY_CHUNK_SHIFT, >= 2)
@@ -455,7 +455,7 @@ uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out,
 
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
                 uint64_t* gains_out, double* kernel_ms) {
-  greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, false);
+  greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, 1);
   return greedy_collect(ctx, 0, k, seeds_out, gains_out, kernel_ms);
 }
 
