@@ -137,6 +137,7 @@ struct GreedyArgs {
   uint32_t* seeds;
   unsigned long long* gains;
   unsigned long long* dbg;      // development: per-pick timestamps (nullable)
+  unsigned long long* dbgb;     // development: every block's barrier arrivals (2 per pick and block)
   // chunked argmax (nc >= chunk_min): chunk_key[c] = the maximum key of
   // chunk c's candidates, refreshed only for the chunks whose counts a
   // cover touched (dirty[c]); the argmax then reads one key per chunk
@@ -207,6 +208,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
       for (uint32_t c = cb0 + threadIdx.x; c < cb1; c += GB) km = umax64(km, a.chunk_key[c]);
       km = block_max(km, red);
       if (threadIdx.x == 0) a.blockmax[blockIdx.x] = km;
+      if (a.dbgb && threadIdx.x == 0) a.dbgb[(2ull * j) * gridDim.x + blockIdx.x] = gtimer_ns();
       grid.sync();
       if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 1] = gtimer_ns();
       km = 0;
@@ -224,6 +226,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
     }
     km = block_max(km, red);
     if (threadIdx.x == 0) a.blockmax[blockIdx.x] = km;
+    if (a.dbgb && threadIdx.x == 0) a.dbgb[(2ull * j) * gridDim.x + blockIdx.x] = gtimer_ns();
     grid.sync();
     if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 1] = gtimer_ns();
     km = 0;
@@ -294,6 +297,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
       if (threadIdx.x == 0) nbig = 0;
     }
     if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j + 2] = gtimer_ns();
+    if (a.dbgb && threadIdx.x == 0) a.dbgb[(2ull * j + 1) * gridDim.x + blockIdx.x] = gtimer_ns();
     grid.sync();
   }
 }
@@ -404,10 +408,13 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   a.chunk_min = cm ? (uint32_t)strtoul(cm, nullptr, 10) : CHUNK_MIN_DEFAULT;
   a.chunk_shift = chunk_shift;
   a.dbg = nullptr;
+  a.dbgb = nullptr;
   const char* gdbg = getenv("EIM_DEBUG_GREEDY");
+  const uint64_t dbg_words = (uint64_t)k * 3 + (uint64_t)k * 2 * blocks;
   if (gdbg && slot == 0) {
-    ctx->stage_a.reserve((uint64_t)k * 24 + 64, false, st);
+    ctx->stage_a.reserve(dbg_words * 8 + 64, false, st);
     a.dbg = ctx->stage_a.as<unsigned long long>();
+    a.dbgb = a.dbg + (uint64_t)k * 3;
   }
   void* args[] = {&a};
   if (!S.ev[0])
@@ -416,9 +423,12 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
   EIM_CUDA(cudaEventRecord(S.ev[1], st));
   ctx->kernel_launches += 2;
-  if (a.dbg) {
-    std::vector<unsigned long long> hd((size_t)k * 3);
-    EIM_CUDA(cudaMemcpyAsync(hd.data(), a.dbg, (size_t)k * 24, cudaMemcpyDeviceToHost, st));
+  if (a.dbg) {  // file: k, blocks, stamps per pick and block, block 0's stamps, every block's arrivals
+    std::vector<unsigned long long> hd(dbg_words + 3);
+    hd[0] = k;
+    hd[1] = blocks;
+    hd[2] = 2;
+    EIM_CUDA(cudaMemcpyAsync(hd.data() + 3, a.dbg, dbg_words * 8, cudaMemcpyDeviceToHost, st));
     EIM_CUDA(cudaStreamSynchronize(st));
     FILE* f = fopen(gdbg, "ab");
     if (f) {

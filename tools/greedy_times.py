@@ -1,5 +1,8 @@
-"""Per-pick phase times of the greedy kernel (EIM_DEBUG_GREEDY timers): argmax
-(to the first grid barrier), cover (to the second), per NodeSelection.
+"""Per-pick phase times of the greedy pick kernel (EIM_DEBUG_GREEDY timers,
+record-index kernel greedy2_kernel): argmax + first barrier, cover, second
+barrier (block 0's stamps), and the spread of the blocks' arrivals at each
+barrier (first to last arrival = how long the barrier waits for the slowest
+block), per NodeSelection of slot 0.
     python tools/greedy_times.py CFG"""
 import os
 import sys
@@ -21,13 +24,30 @@ if os.path.exists(path):
     os.remove(path)
 os.environ["EIM_DEBUG_GREEDY"] = path
 eim.eim_imm_run(ctx, g, c["k"], c["eps"], c["ell"], c["model"], 1)
-t = np.fromfile(path, dtype=np.uint64).astype(np.int64).reshape(-1, 3)
-k = c["k"]
-for r in range(len(t) // k):
-    b = t[r * k:(r + 1) * k]
+raw = np.fromfile(path, dtype=np.uint64).astype(np.int64)
+pos, r = 0, 0
+while pos < len(raw):
+    k, nb, pp = int(raw[pos]), int(raw[pos + 1]), int(raw[pos + 2])
+    pos += 3
+    b = raw[pos:pos + 3 * k].reshape(k, 3)
+    pos += 3 * k
+    arr = raw[pos:pos + pp * k * nb].reshape(k, pp, nb)
+    pos += pp * k * nb
     arg = (b[:, 1] - b[:, 0]) / 1e3
     cov = (b[:, 2] - b[:, 1]) / 1e3
     nxt = (b[1:, 0] - b[:-1, 2]) / 1e3
-    print(f"{cfg} selection {r}: picks {k} total {(b[-1, 2] - b[0, 0]) / 1e3:.1f} us; argmax+sync median {np.median(arg):.2f} "
-          f"max {arg.max():.2f}; cover median {np.median(cov):.2f} max {cov.max():.2f} (first {cov[0]:.2f}); "
-          f"second sync median {np.median(nxt) if len(nxt) else 0:.2f} us")
+    s1 = (arr[:, 0].max(1) - arr[:, 0].min(1)) / 1e3   # argmax arrivals spread
+    s2 = (arr[:, 1].max(1) - arr[:, 1].min(1)) / 1e3   # cover arrivals spread
+    l1 = (b[:, 1] - arr[:, 0].max(1)) / 1e3            # last arrival -> block 0 leaves barrier 1
+    l2 = (b[1:, 0] - arr[:-1, 1].max(1)) / 1e3          # last arrival -> block 0 leaves barrier 2
+    print(f"{cfg} selection {r} ({nb} blocks): {k} picks in {(b[-1, 2] - b[0, 0]) / 1e3:.1f} us = "
+          f"{(b[-1, 2] - b[0, 0]) / 1e3 / k:.2f} us/pick | argmax+B1 med {np.median(arg):.2f} | "
+          f"cover med {np.median(cov):.2f} (first {cov[0]:.2f}) | B2 med {np.median(nxt) if len(nxt) else 0:.2f} | "
+          f"arrival spread B1 med {np.median(s1):.2f} B2 med {np.median(s2):.2f} | "
+          f"last-arrival->exit B1 med {np.median(l1):.2f} B2 med {np.median(l2) if len(l2) else 0:.2f} us")
+    if pp == 4:  # per block: B2 exit -> scan done, and the spread of the B2 exits
+        sc = (arr[:, 3] - arr[:, 2]) / 1e3
+        ex = (arr[:, 2].max(1) - arr[:, 2].min(1)) / 1e3
+        print(f"    per-block scan med {np.median(sc):.2f} max-over-blocks med {np.median(sc.max(1)):.2f} | "
+              f"B2-exit spread med {np.median(ex):.2f} | scan-done -> B1 arrival med {np.median((arr[:, 0] - arr[:, 3]) / 1e3):.2f} us")
+    r += 1
