@@ -292,7 +292,8 @@ def main():
                    "us_per_pick": (g_ms * 1e3 / g_picks) if g_picks else None,
                    "selections_per_imm": stats[-1]["select_launches"], "picks_per_imm": stats[-1]["select_picks"],
                    "kernel_ms_per_imm": g_ms / args.steps,
-                   "note": "two concurrent selections (paired rounds) both count their device time"}
+                   "note": "concurrent selections (the rounds one sampler launch covers) each count their "
+                           "device time"}
 
     # end to end through the public API with host buffers: H2D of the graph
     # from pinned memory + IMM + D2H of the result, every step

@@ -271,8 +271,20 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
 // consume_all (RF_DROP_EMPTY, use = every non-empty set of the launch): all
 // ids of the launch count as consumed (a multi-rank round whose cut lies on
 // a later rank).
+// cuts (plain rounds, one GPU): the append also leaves, for each cut j,
+// snap[j] = C over the sets up to s_local cut[j] (C from before the append
+// plus those sets' members) and total[j] = the arena elements up to that
+// set -- the inputs of the run-ahead selections of the rounds the append
+// covers, in one scan, one host read-back and one scatter instead of one per
+// round.
+struct AppendCuts {
+  uint32_t n = 0;        // <= 2
+  uint64_t cut[2] = {};  // s_local, from < cut < use
+  uint32_t* snap[2] = {};
+  uint64_t total[2] = {};  // out
+};
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from = 0,
-                            bool keep = false, bool consume_all = false);
+                            bool keep = false, bool consume_all = false, AppendCuts* cuts = nullptr);
 // RF_DROP_EMPTY rounds: wait, drop the roots and count the non-empty sets
 // of the whole launch (idempotent; round_finalize then keeps the first `use`).
 uint64_t round_elim_kept(eim_ctx* ctx, const eim_graph* g, Round& rd);
@@ -327,6 +339,12 @@ void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_
 void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t concurrent);
 uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
                         double* kernel_ms = nullptr);
+
+// development (EIM_TRACE=1): host timestamps of the IMM phases on stderr,
+// in ms since the last trace_reset (marks after a host synchronisation
+// approximate the device's completion time)
+void trace_reset();
+void trace_mark(const char* what, uint64_t a = 0, uint64_t b = 0);
 
 // ---- imm.cpp
 void imm_params(uint32_t n, uint32_t k, double eps, double ell, eim_imm_params_t* out);

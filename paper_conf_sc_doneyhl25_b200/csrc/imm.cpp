@@ -42,6 +42,9 @@ double ms_since(clk::time_point t0) {
   return std::chrono::duration<double, std::milli>(clk::now() - t0).count();
 }
 
+clk::time_point trace_t0;
+bool trace_on = false;
+
 struct Exchange {
   DevBuf counts, offs_recv, mem_recv;
 };
@@ -181,6 +184,41 @@ class RoundSampler {
   // the held lookahead launch can supply sets [from, to) without a launch
   bool holds(uint64_t from, uint64_t to) const { return held_ && held_done_ == from && launch_end_ >= to; }
 
+  // One GPU, plain runs: can [R, to) come from one launch (held or new)?
+  bool can_multi(uint64_t R, uint64_t to) const {
+    return W() == 1 && !elim_ && !speculate_ && lookahead_ &&
+           (holds(R, to) || to - R <= max_launch_ids(ctx_));
+  }
+
+  // Sets [R, ends.back()) from one launch, appended in one pass; for every
+  // earlier end t the append leaves snaps[t] = C over sets [0, ends[t]) and
+  // totals[t] = the arena elements up to ends[t] (run-ahead selections).
+  void grow_multi(uint64_t& R, const std::vector<uint64_t>& ends, uint32_t* const* snaps,
+                  std::vector<uint64_t>& totals) {
+    const auto t0 = clk::now();
+    const uint64_t to = ends.back();
+    st_->ids_sampled += to - R;
+    if (!holds(R, to)) {
+      drop_held();
+      launch_range(R, to);
+    }
+    AppendCuts cuts;
+    cuts.n = (uint32_t)ends.size() - 1;
+    if (cuts.n > 2) fail(EIM_E_STATE, "grow_multi: at most three rounds per append");
+    for (uint32_t j = 0; j < cuts.n; ++j) {
+      cuts.cut[j] = ends[j] - launch_first_;
+      cuts.snap[j] = snaps[j];
+    }
+    Round& rd = ctx_->rounds[0];
+    account(round_finalize(ctx_, g_, rd, to - launch_first_, R - launch_first_, to < launch_end_, false, &cuts));
+    totals.assign(cuts.total, cuts.total + cuts.n);
+    totals.push_back(arena_cursor(ctx_));
+    held_done_ = to;
+    if (to >= launch_end_) drop_held();
+    R = to;
+    st_->ms_sample += ms_since(t0);
+  }
+
   void cancel() {
     if (spec_) {
       round_cancel(ctx_, *spec_);
@@ -233,6 +271,7 @@ class RoundSampler {
     launch_first_ = R;
     launch_end_ = end;
     eim_shard_range(R, end - R, ctx_->rank, W(), &my_lo_, &my_hi_);
+    trace_mark("launch", first, end);
     Round& rd = ctx_->rounds[0];
     if (my_hi_ > my_lo_)
       round_launch(ctx_, g_, model_, seed_, id_base_ + my_lo_, my_hi_ - my_lo_, id_base_, W() == 1, rd, stream_of(rd),
@@ -376,10 +415,22 @@ class RoundSampler {
 
 }  // namespace
 
+void trace_reset() {
+  trace_on = std::getenv("EIM_TRACE") != nullptr;
+  trace_t0 = clk::now();
+}
+
+void trace_mark(const char* what, uint64_t a, uint64_t b) {
+  if (!trace_on) return;
+  std::fprintf(stderr, "trace %9.3f ms  %s %llu %llu\n", ms_since(trace_t0), what, (unsigned long long)a,
+               (unsigned long long)b);
+}
+
 void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double ell, eim_model model,
              uint64_t seed, uint32_t flags, uint32_t* seeds_out, uint64_t* theta_out, double* spread_out,
              eim_stats* st) {
   const auto t_start = clk::now();
+  trace_reset();
   const uint32_t n = g->view.n;
   const bool elim = (flags & EIM_F_SOURCE_ELIM) != 0, fresh = (flags & EIM_F_FRESH_FINAL) != 0;
   if (elim && !graph_has_proper_edge(ctx, g))
@@ -448,29 +499,17 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
           J = i + 1;
           if (pairing && has_round(i + 2) && continues(i) && continues(i + 1)) J = i + 2;
         }
-        sampler.grow(R, theta_round(i), theta_round(J));
-        R_sel = R;
-        const auto ts = clk::now();
-        if (pairing && J > i && sampler.holds(R, theta_round(i + 1))) {
-          const uint32_t nsel = J - i + 1;
-          std::vector<uint64_t> Rs(nsel), totals(nsel);
-          DevBuf* snaps[2] = {&ctx->C_snap, &ctx->C_snap2};
-          for (uint32_t t = 0; t < nsel; ++t) {
-            Rs[t] = R;
-            totals[t] = arena_cursor(ctx);
-            if (t + 1 == nsel) break;
-            snaps[t]->reserve((uint64_t)n * sizeof(uint32_t), false, s);
-            EIM_CUDA(cudaMemcpyAsync(snaps[t]->p, ctx->C_total.p, (uint64_t)n * sizeof(uint32_t),
-                                     cudaMemcpyDeviceToDevice, s));
-            const auto tg = clk::now();
-            sampler.grow(R, theta_round(i + t + 1), theta_round(J));  // appends the held sets, no launch
-            st->ms_select -= ms_since(tg);
-          }
-          // slot nsel-1-t runs round i+t (round J, on the live counts, in slot 0)
+        // run the selections of rounds i..i+nsel-1 at once: slot nsel-1-t
+        // runs round i+t on Rs[t] sets (arena prefix totals[t]) with C
+        // snapshot t (round J on the live counts, in slot 0); the later
+        // rounds' results wait in `pre`
+        auto run_ahead = [&](uint32_t nsel, const std::vector<uint64_t>& Rs, const std::vector<uint64_t>& totals,
+                             uint32_t* const* snaps) {
           for (uint32_t t = 0; t < nsel; ++t)
             greedy_setup(ctx, nsel - 1 - t, n, Rs[t], totals[t],
-                         t + 1 == nsel ? ctx->C_total.as<uint32_t>() : snaps[t]->as<uint32_t>());
+                         t + 1 == nsel ? ctx->C_total.as<uint32_t>() : snaps[t]);
           for (uint32_t t = 0; t < nsel; ++t) greedy_picks(ctx, nsel - 1 - t, n, Rs[t], k, nsel);
+          trace_mark("selections enqueued", nsel, Rs[nsel - 1]);
           for (uint32_t t = 0; t < nsel; ++t) {
             if (t == 0) {
               cov = greedy_collect(ctx, nsel - 1, k, S.data(), nullptr, &st->ms_select_kernel);
@@ -480,14 +519,57 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
               pre.push_back(std::move(q));
             }
           }
+          trace_mark("selections collected", nsel, Rs[nsel - 1]);
           st->select_launches += nsel;
           st->select_picks += (uint64_t)nsel * k;
+        };
+        DevBuf* snapb[2] = {&ctx->C_snap, &ctx->C_snap2};
+        const uint32_t nsel = J - i + 1;
+        if (pairing && J > i && sampler.can_multi(R, theta_round(J))) {
+          // rounds i..J from one launch and ONE append (one scan, one host
+          // read-back, one scatter that also fills the round snapshots of C)
+          std::vector<uint64_t> Rs(nsel), totals;
+          uint32_t* snaps[2] = {nullptr, nullptr};
+          for (uint32_t t = 0; t < nsel; ++t) Rs[t] = theta_round(i + t);
+          for (uint32_t t = 0; t + 1 < nsel; ++t) {
+            snapb[t]->reserve((uint64_t)n * sizeof(uint32_t), false, s);
+            snaps[t] = snapb[t]->as<uint32_t>();
+          }
+          sampler.grow_multi(R, Rs, snaps, totals);
+          R_sel = Rs[0];
+          const auto ts = clk::now();
+          run_ahead(nsel, Rs, totals, snaps);
+          st->ms_select += ms_since(ts);
         } else {
-          cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
-          st->select_launches += 1;
-          st->select_picks += k;
+          sampler.grow(R, theta_round(i), theta_round(J));
+          R_sel = R;
+          const auto ts = clk::now();
+          if (pairing && J > i && sampler.holds(R, theta_round(i + 1))) {
+            // (a launch split for the table budget) one append per round
+            std::vector<uint64_t> Rs(nsel), totals(nsel);
+            uint32_t* snaps[2] = {nullptr, nullptr};
+            for (uint32_t t = 0; t < nsel; ++t) {
+              Rs[t] = R;
+              totals[t] = arena_cursor(ctx);
+              if (t + 1 == nsel) break;
+              snapb[t]->reserve((uint64_t)n * sizeof(uint32_t), false, s);
+              snaps[t] = snapb[t]->as<uint32_t>();
+              EIM_CUDA(cudaMemcpyAsync(snaps[t], ctx->C_total.p, (uint64_t)n * sizeof(uint32_t),
+                                       cudaMemcpyDeviceToDevice, s));
+              const auto tg = clk::now();
+              sampler.grow(R, theta_round(i + t + 1), theta_round(J));  // appends the held sets, no launch
+              st->ms_select -= ms_since(tg);
+            }
+            run_ahead(nsel, Rs, totals, snaps);
+          } else {
+            trace_mark("selection", R);
+            cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
+            trace_mark("selection collected", R);
+            st->select_launches += 1;
+            st->select_picks += k;
+          }
+          st->ms_select += ms_since(ts);
         }
-        st->ms_select += ms_since(ts);
       }
       R_selected = R_sel;
       if (st->rounds < 64) {
@@ -538,6 +620,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   }
   if (R != R_selected) {  // NodeSelection is deterministic: reuse the last run on the same R
     const auto ts = clk::now();
+    trace_mark("final selection", R);
     cov = greedy(ctx, n, R, k, S.data(), nullptr, &st->ms_select_kernel);
     st->select_launches += 1;
     st->select_picks += k;
@@ -553,6 +636,7 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
   if (spread_out) *spread_out = (double)n * (double)cov / (double)R;
   st->kernel_launches = ctx->kernel_launches - launches0;
   st->ms_total = ms_since(t_start);
+  trace_mark("imm done", R);
 }
 
 }  // namespace eim

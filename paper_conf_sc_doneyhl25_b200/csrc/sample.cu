@@ -169,6 +169,7 @@ struct RoundView {
   unsigned long long* qc;        // task queue q: head at qc[16 q], tail at qc[16 q + 1] (one 128-B line each)
   uint32_t prefetch;             // L2-prefetch in_nbr of parked live edges (EIM_NO_PREFETCH=1 turns it off)
   const uint32_t* list;          // IC: ticket t -> s_local (the ids whose root has in-edges; root pre-pass)
+  uint32_t lt_evict;             // LT walk-store loads marked evict-first in L2 (EIM_LT_NO_EVICT=1: default policy)
 };
 
 // Split-off tasks go to TQ queues (descriptor segments of tcap / TQ each):
@@ -986,9 +987,20 @@ __device__ __forceinline__ int table_resolve(unsigned long long* keys, uint32_t 
 // insert of the current vertex is resolved, so a step costs one memory round
 // trip.  When the current vertex turns out to be a revisit (the walk stops,
 // P:136), the speculative insert is overwritten with TABLE_TOMB.
+__device__ __forceinline__ uint4 aug_load(const uint4* p, unsigned long long pol) {
+  if (pol == 0ull) return __ldg(p);
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p), "l"(pol));
+  return r;
+}
+
 __global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* __restrict__ aug, RoundView R,
                                                      uint64_t count, SampleCtl* ctl) {
   const PhiloxKey& K = R.K;
+  unsigned long long pol = 0ull;  // L2 policy of the walk-store loads (0: default)
+  if (R.lt_evict) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
   unsigned long long edges_acc = 0;
   for (;;) {
     const volatile unsigned int* cp = R.cancel;
@@ -1006,7 +1018,7 @@ __global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* _
     unsigned long long steps = 0;
     if (ok && d) {
       // the step from the root: entry a -> vertex v (insert pending), nx = the entry chosen from v
-      const uint4 a = __ldg(aug + e0 + __umul64hi((unsigned long long)tau << 32, d));
+      const uint4 a = aug_load(aug + e0 + __umul64hi((unsigned long long)tau << 32, d), pol);
       steps = 1;
       uint32_t v = a.x;
       unsigned long long key = table_key(s_local, v);
@@ -1016,7 +1028,7 @@ __global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* _
       uint4 nx = a;
       if (nxt) {
         const uint32_t tv = word_of(philox_at((uint64_t)(v >> 2), s, TAG_LT, K), v & 3u);
-        nx = __ldg(aug + ((uint64_t)a.z | ((uint64_t)a.w << 32)) + __umul64hi((unsigned long long)tv << 32, a.y));
+        nx = aug_load(aug + ((uint64_t)a.z | ((uint64_t)a.w << 32)) + __umul64hi((unsigned long long)tv << 32, a.y), pol);
       }
       for (;;) {
         // speculate the step from v: v2 = nx.x, its insert and the entry chosen from v2
@@ -1032,7 +1044,8 @@ __global__ void __launch_bounds__(256) lt_aug_kernel(GraphView g, const uint4* _
           nxt2 = nx.y != 0u;
           if (nxt2) {
             const uint32_t tv2 = word_of(philox_at((uint64_t)(v2 >> 2), s, TAG_LT, K), v2 & 3u);
-            nx2 = __ldg(aug + ((uint64_t)nx.z | ((uint64_t)nx.w << 32)) + __umul64hi((unsigned long long)tv2 << 32, nx.y));
+            nx2 = aug_load(aug + ((uint64_t)nx.z | ((uint64_t)nx.w << 32)) + __umul64hi((unsigned long long)tv2 << 32, nx.y),
+                           pol);
           }
         }
         // resolve v's insert
@@ -1162,7 +1175,9 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
                                uint32_t use,
                                uint32_t* __restrict__ fill, uint32_t* __restrict__ arena, uint32_t ab,
                                uint32_t* __restrict__ C, GV g, bool ic, unsigned long long* __restrict__ esum,
-                               const uint32_t* __restrict__ roots, const uint32_t* __restrict__ kidx) {
+                               const uint32_t* __restrict__ roots, const uint32_t* __restrict__ kidx,
+                               uint32_t* __restrict__ snap0, uint32_t cut0, uint32_t* __restrict__ snap1,
+                               uint32_t cut1) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   unsigned long long e = 0;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nslots; i += stride) {
@@ -1177,6 +1192,8 @@ __global__ void scatter_kernel(const unsigned long long* __restrict__ keys, uint
     const uint32_t p = atomicAdd(&fill[s_local], 1u);
     arena_put(arena, set_start[si] + p, ab, v);
     if (C) atomicAdd(&C[v], 1u);
+    if (snap0 && s_local < cut0) atomicAdd(&snap0[v], 1u);  // round snapshots (AppendCuts)
+    if (snap1 && s_local < cut1) atomicAdd(&snap1[v], 1u);
   }
   if (ic) {
     for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(FULL, e, o);
@@ -1340,7 +1357,8 @@ static RoundView round_view(Round& rd) {
                    std::getenv("EIM_NO_HOIST") ? 1u : 0u,
                    round_queues(rd),
                    std::getenv("EIM_NO_PREFETCH") ? 0u : 1u,
-                   rd.list.as<uint32_t>()};
+                   rd.list.as<uint32_t>(),
+                   std::getenv("EIM_LT_NO_EVICT") ? 0u : 1u};
 }
 
 // one sampler launch over rd's remaining work, bracketed by events
@@ -1466,7 +1484,13 @@ void round_launch(eim_ctx* ctx, const eim_graph* g, eim_model model, uint64_t se
   const double mean = ctx->est_mean_size > 0 ? ctx->est_mean_size : 64.0;
   // EIM_TABLE_BITS: smallest table (tests force overflow and the redo path)
   uint32_t bits = std::min<uint32_t>(std::max<uint32_t>(env_u32("EIM_TABLE_BITS", 20), 4), 31);
-  while (bits < 31 && (double)(1ull << bits) < 4.0 * mean * (double)count) bits++;
+  const char* tf = std::getenv("EIM_TABLE_FACTOR");  // development: slots per expected member (default 4)
+  const double factor = tf ? std::max(1.1, std::strtod(tf, nullptr)) : 4.0;
+  while (bits < 31 && (double)(1ull << bits) < factor * mean * (double)count) bits++;
+  // LT: twice as many slots while the table stays within the 2^30-slot
+  // launch budget (fewer probe collisions on the walk's critical path: C3
+  // walk kernel 0.963 -> 0.869 ms; 4x more cost the scatter more than it saves)
+  if (model == EIM_LT && !tf && bits < 30) bits++;
   rd.bits = bits;
   round_start(ctx, g, rd, st, spare_sm_slot);
 }
@@ -1501,6 +1525,7 @@ static void round_wait(eim_ctx* ctx, const eim_graph* g, Round& rd) {
       EIM_CUDA(cudaMemcpyAsync(h, ctl, sizeof(SampleCtl), cudaMemcpyDeviceToHost, st));
       EIM_CUDA(cudaStreamSynchronize(st));
       const uint64_t ntk = rd.model == EIM_IC ? h->ntickets : rd.count;
+      trace_mark("sampler done", rd.first, rd.count);
       if ((h->ticket >= ntk && h->outstanding == 0) || h->arena_fail) break;
       round_resume(ctx, g, rd, st);
     }
@@ -1573,7 +1598,7 @@ uint64_t round_elim_kept(eim_ctx* ctx, const eim_graph* g, Round& rd) {
 }
 
 SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_t use, uint64_t from, bool keep,
-                            bool consume_all) {
+                            bool consume_all, AppendCuts* cuts) {
   SampleResult res;
   if (!rd.launched || rd.count == 0) return res;
   if (use > rd.count || from > use) fail(EIM_E_STATE, "round_finalize beyond the launched range");
@@ -1671,8 +1696,24 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     EIM_CUDA(cudaGetLastError());
   }
   EIM_CUDA(cudaMemcpyAsync(&h->ticket, excl + nsets, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  const uint32_t ncut = cuts ? cuts->n : 0u;
+  uint64_t* hcut = reinterpret_cast<uint64_t*>(static_cast<char*>(ctx->h_pinned) + 3600);
+  if (ncut) {
+    if (ncut > 2 || drop_root || !rd.hist) fail(EIM_E_STATE, "append cuts need a plain round with its histogram");
+    for (uint32_t j = 0; j < ncut; ++j) {
+      if (cuts->cut[j] <= from || cuts->cut[j] >= use) fail(EIM_E_STATE, "append cut outside the appended range");
+      EIM_CUDA(cudaMemcpyAsync(hcut + j, excl + (cuts->cut[j] - from), sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+    }
+  }
   EIM_CUDA(cudaStreamSynchronize(st));
   const uint64_t total = h->ticket, cursor = ctx->arena_used;
+  for (uint32_t j = 0; j < ncut; ++j) {
+    cuts->total[j] = cursor + hcut[j];
+    // the snapshot starts as C before this append; the scatter adds the sets below the cut
+    EIM_CUDA(cudaMemcpyAsync(cuts->snap[j], ctx->C_total.p, (uint64_t)g->view.n * sizeof(uint32_t),
+                             cudaMemcpyDeviceToDevice, st));
+  }
+  trace_mark("append sizes", from, use);
   arena_ensure(ctx, cursor + total);
   if (nsets) {
     place_sets_kernel<<<grid_for(ctx, nsets, 256), 256, 0, st>>>(excl, sizes, nsets, cursor, set_index0 + from,
@@ -1685,7 +1726,9 @@ SampleResult round_finalize(eim_ctx* ctx, const eim_graph* g, Round& rd, uint64_
     scatter_kernel<<<grid_for(ctx, nslots, 256), 256, 0, st>>>(
         rd.table.as<unsigned long long>(), nslots, ctx->set_start.as<uint64_t>(), set_index0,
         (uint32_t)from, (uint32_t)consumed, rd.fill.as<uint32_t>(), ctx->arena.as<uint32_t>(), ctx->arena_b,
-        rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_acc, roots, kidx);
+        rd.hist ? ctx->C_total.as<uint32_t>() : nullptr, gv, ic, d_edges_acc, roots, kidx,
+        ncut > 0 ? cuts->snap[0] : nullptr, ncut > 0 ? (uint32_t)cuts->cut[0] : 0u,
+        ncut > 1 ? cuts->snap[1] : nullptr, ncut > 1 ? (uint32_t)cuts->cut[1] : 0u);
   };
   with_graph_view(g, scatter);
   EIM_CUDA(cudaGetLastError());

@@ -360,14 +360,18 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   uint32_t* pos = S.inv_fill.as<uint32_t>();
   uint64_t* inv_off = S.inv_off.as<uint64_t>();
   // ---- 3. the k picks in one cooperative kernel
-  S.covered.reserve(std::max<uint64_t>(num_sets, 1), false, st);
-  S.selected.reserve((uint64_t)n + 4, false, st);
+  // covered flags (num_sets), selected flags (n), the all-covered cursor:
+  // one buffer, one memset
+  const uint64_t fl_sets = (std::max<uint64_t>(num_sets, 1) + 15) & ~15ull;
+  const uint64_t fl_sel = ((uint64_t)n + 4 + 15) & ~15ull;
+  S.covered.reserve(fl_sets + fl_sel + 16, false, st);
   S.seeds.reserve((uint64_t)k * sizeof(uint32_t), false, st);
   S.gains.reserve((uint64_t)k * sizeof(unsigned long long), false, st);
-  EIM_CUDA(cudaMemsetAsync(S.covered.p, 0, std::max<uint64_t>(num_sets, 1), st));
-  EIM_CUDA(cudaMemsetAsync(S.selected.p, 0, (uint64_t)n + 4, st));
-  int per_sm = 0;
-  EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
+  EIM_CUDA(cudaMemsetAsync(S.covered.p, 0, fl_sets + fl_sel + 16, st));
+  uint8_t* selected = S.covered.as<uint8_t>() + fl_sets;
+  uint32_t* zc = reinterpret_cast<uint32_t*>(selected + fl_sel);
+  static int per_sm = 0;  // occupancy of the pick kernel (a property of the binary and the device)
+  if (per_sm == 0) EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
   const char* gbe = getenv("EIM_GREEDY_BLOCKS");  // development: grid of the greedy kernel
   uint32_t blocks = gbe ? (uint32_t)atoi(gbe) : (uint32_t)ctx->sm_count;
   // two concurrent selections get half the SMs each: measured on C3 (both
@@ -384,9 +388,7 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   const uint64_t nchunks_max = ((uint64_t)n >> chunk_shift) + 2;
   S.best.reserve(((uint64_t)blocks + nchunks_max + 8) * sizeof(unsigned long long) + 64, false, st);
   S.dirty.reserve(nchunks_max, false, st);
-  EIM_CUDA(cudaMemsetAsync(S.dirty.p, 1, nchunks_max, st));  // every chunk key is computed at the first pick
-  uint32_t* zc = reinterpret_cast<uint32_t*>(S.best.as<unsigned long long>() + blocks);
-  EIM_CUDA(cudaMemsetAsync(zc, 0, sizeof(uint32_t), st));
+  if (cm) EIM_CUDA(cudaMemsetAsync(S.dirty.p, 1, nchunks_max, st));  // every chunk key is computed at the first pick
   GreedyArgs a;
   a.k = k;
   a.nc = pos + n;
@@ -399,7 +401,7 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   a.set_len = ctx->set_len.as<uint32_t>();
   a.arena_c = S.arena_c.as<uint32_t>();
   a.blockmax = S.best.as<unsigned long long>();
-  a.selected = S.selected.as<uint8_t>();
+  a.selected = selected;
   a.zc = zc;
   a.seeds = S.seeds.as<uint32_t>();
   a.gains = S.gains.as<unsigned long long>();
