@@ -330,13 +330,14 @@ uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_
 // stream first), then wait and read the result.  C and the arena prefix must
 // stay unchanged until greedy_collect.
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
-                   uint32_t k, uint32_t concurrent);
+                   uint32_t k);
 // greedy_launch in two halves, so two slots' setups can overlap before the
 // host reads their candidate counts
 void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C);
-// concurrent: the number of selections running at the same time (each
-// gets that share of the SMs)
-void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t concurrent);
+// blocks_share: the blocks of this selection when several run at the same
+// time (greedy_shares), 0 = one per SM
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t blocks_share);
+void greedy_shares(eim_ctx* ctx, uint32_t nsel, const uint64_t* num_sets, uint32_t* blocks);
 uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out, uint64_t* gains_out,
                         double* kernel_ms = nullptr);
 

@@ -508,7 +508,9 @@ void imm_run(eim_ctx* ctx, const eim_graph* g, uint32_t k, double eps, double el
           for (uint32_t t = 0; t < nsel; ++t)
             greedy_setup(ctx, nsel - 1 - t, n, Rs[t], totals[t],
                          t + 1 == nsel ? ctx->C_total.as<uint32_t>() : snaps[t]);
-          for (uint32_t t = 0; t < nsel; ++t) greedy_picks(ctx, nsel - 1 - t, n, Rs[t], k, nsel);
+          uint32_t share[3];
+          greedy_shares(ctx, nsel, Rs.data(), share);
+          for (uint32_t t = 0; t < nsel; ++t) greedy_picks(ctx, nsel - 1 - t, n, Rs[t], k, share[t]);
           trace_mark("selections enqueued", nsel, Rs[nsel - 1]);
           for (uint32_t t = 0; t < nsel; ++t) {
             if (t == 0) {

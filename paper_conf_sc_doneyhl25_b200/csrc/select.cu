@@ -18,6 +18,8 @@
 //      pick is the lowest unselected vertex id (R10).
 #include <cooperative_groups.h>
 
+#include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -305,9 +307,9 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
 }  // namespace
 
 void greedy_launch(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_t total, const uint32_t* C,
-                   uint32_t k, uint32_t concurrent) {
+                   uint32_t k) {
   greedy_setup(ctx, slot, n, num_sets, total, C);
-  greedy_picks(ctx, slot, n, num_sets, k, concurrent);
+  greedy_picks(ctx, slot, n, num_sets, k, 0);
 }
 
 // steps 1-2: candidates, remapped arena, inverted index (enqueued on the slot's stream)
@@ -353,8 +355,34 @@ void greedy_setup(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint64_
   ctx->kernel_launches += 7;
 }
 
+// Blocks of nsel concurrent selections over num_sets[t] sets each: the SMs
+// are shared in proportion to sqrt(num_sets) (a larger R has more
+// candidates to scan and longer lists to cover, every selection runs k
+// picks, and a pick's latency falls slowly with its blocks), at least 16
+// blocks each.  Measured against an even split: C3 selection 1.465 -> 1.41
+// ms, C2 1.675 -> 1.65 ms (weights R^1: 1.42 / 1.66, R^1.5: 1.51 / 1.72).
+// EIM_GREEDY_EVEN=1: an even split.
+void greedy_shares(eim_ctx* ctx, uint32_t nsel, const uint64_t* num_sets, uint32_t* blocks) {
+  const uint32_t sm = (uint32_t)ctx->sm_count, lo = std::min<uint32_t>(16, sm / std::max(nsel, 1u));
+  const char* pe = getenv("EIM_GREEDY_POW");  // development: weights num_sets^pow (0: even)
+  const double pw = getenv("EIM_GREEDY_EVEN") ? 0.0 : (pe ? std::strtod(pe, nullptr) : 0.5);
+  double tot = 0;
+  for (uint32_t t = 0; t < nsel; ++t) tot += std::pow((double)std::max<uint64_t>(num_sets[t], 1), pw);
+  uint32_t used = 0;
+  for (uint32_t t = 0; t < nsel; ++t) {
+    const double w = std::pow((double)std::max<uint64_t>(num_sets[t], 1), pw) / tot;
+    blocks[t] = std::max(lo, (uint32_t)(w * sm));
+    used += blocks[t];
+  }
+  while (used > sm) {  // the minimum pushed the sum over: take from the largest share
+    uint32_t* b = std::max_element(blocks, blocks + nsel);
+    --*b;
+    --used;
+  }
+}
+
 // step 3: the k picks in one cooperative grid kernel
-void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t concurrent) {
+void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t blocks_share) {
   GreedySlot& S = ctx->gs[slot];
   cudaStream_t st = S.stream;
   uint32_t* pos = S.inv_fill.as<uint32_t>();
@@ -374,11 +402,10 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   if (per_sm == 0) EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
   const char* gbe = getenv("EIM_GREEDY_BLOCKS");  // development: grid of the greedy kernel
   uint32_t blocks = gbe ? (uint32_t)atoi(gbe) : (uint32_t)ctx->sm_count;
-  // two concurrent selections get half the SMs each: measured on C3 (both
-  // selections of the paired rounds 1 and 2), 74 + 74 blocks take 1.33 ms
-  // against 1.93 ms for the two one after the other on 148 blocks, while
-  // two 148-block grids launched together take 2.0 ms (they do not overlap)
-  if (concurrent > 1) blocks = std::max(1u, blocks / concurrent);
+  // concurrent selections get their share of the SMs (greedy_shares): two
+  // 148-block cooperative grids launched together do not overlap (C3: 2.0 ms
+  // against 1.93 ms one after the other), 74 + 74 blocks do (1.33 ms)
+  if (blocks_share > 0) blocks = std::min(blocks, blocks_share);
   blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
   // chunked argmax from this many candidates on (EIM_GREEDY_CHUNK_MIN; 0:
   // always) with 2^shift candidates per chunk (EIM_GREEDY_CHUNK_SHIFT, >= 2)
@@ -467,7 +494,7 @@ uint64_t greedy_collect(eim_ctx* ctx, int slot, uint32_t k, uint32_t* seeds_out,
 
 uint64_t greedy(eim_ctx* ctx, uint32_t n, uint64_t num_sets, uint32_t k, uint32_t* seeds_out,
                 uint64_t* gains_out, double* kernel_ms) {
-  greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k, 1);
+  greedy_launch(ctx, 0, n, num_sets, arena_cursor(ctx), ctx->C_total.as<uint32_t>(), k);
   return greedy_collect(ctx, 0, k, seeds_out, gains_out, kernel_ms);
 }
 
