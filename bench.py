@@ -54,6 +54,22 @@ def philox_roof_gwords():
         return 1630.0, "fallback constant", []
 
 
+GATHER_PROBE = os.path.join(ROOT, "tools", "gather_roof", "gather_roof")
+
+
+def gather_roof(walkers):
+    """(steps/s, probe line) of tools/gather_roof --cas at the LT round's
+    concurrency: random dependent 16-B loads over a walk-store-sized buffer
+    plus one table CAS per step -- the roof of a walk step."""
+    try:
+        out = subprocess.run([GATHER_PROBE, "--cas"], capture_output=True, text=True, timeout=120).stdout
+        lines = [json.loads(l) for l in out.splitlines() if l.startswith("{")]
+        best = min(lines, key=lambda l: abs(l["walkers"] - walkers))
+        return best["steps_per_s"], lines
+    except Exception:
+        return None, []
+
+
 def ncu_traffic(model):
     """DRAM bytes per launch of the dominant kernel from the newest committed
     `ncu --set full` summary of this round (profiles/r02_*), else round 1's."""
@@ -284,6 +300,16 @@ def main():
         peak_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in _peaks() else "fallback 8 TB/s"
         achieved = (LT_STEP_BYTES * k_edges_local / k_launch) / (k_ms / k_launch / 1e3) / 1e9 if k_ms > 0 else None
     traffic, traffic_src = ncu_traffic(c["model"])  # DRAM bytes per launch, committed ncu --set full capture
+    lt_ra = None
+    if c["model"] == "LT" and k_ms > 0 and rank == 0:
+        # the walk step is a random dependent access: its roof is the random
+        # dependent-load + CAS rate at the round's concurrency (tools/gather_roof)
+        ra_peak, ra_probe = gather_roof(stats[-1]["theta"])
+        ra_ach = (k_edges_local / k_launch) / (k_ms / k_launch / 1e3)
+        lt_ra = {"achieved_steps_per_s": ra_ach, "peak_steps_per_s": ra_peak,
+                 "frac": (ra_ach / ra_peak) if ra_peak else None, "probe": ra_probe,
+                 "basis": "walk steps/s of lt_aug_kernel vs tools/gather_roof --cas (random dependent 16-B loads "
+                          "over a 1.9-GB buffer + one CAS into a 2^25-slot table per step, same number of walkers)"}
     # the greedy pick kernel: latency-bound (two grid barriers and ~4 dependent
     # L2 round trips per pick), reported as device time per pick
     g_ms = sum(s["ms_select_kernel"] for s in stats)
@@ -424,7 +450,8 @@ def main():
                          {"bound": "hbm", "kernel": "lt_aug_kernel (LT reverse walks on the walk store)", "achieved": achieved,
                           "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
                           "traffic": traffic, "traffic_source": traffic_src,
-                          "peak_basis": f"{LT_STEP_BYTES:.0f} algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6"}),
+                          "peak_basis": f"{LT_STEP_BYTES:.0f} algorithmic bytes per walk step; " + peak_src + "; DESIGN.md §6",
+                          "random_access": lt_ra}),
             "greedy": greedy_line,
             # IC: examined edges/s vs the Philox roof; LT: LT_STEP_BYTES per walk step vs HBM
             "sampler_fixed_budget": (dict(budget, frac=(budget["edges_per_s"] / 1e9 / world / peak)

@@ -82,12 +82,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 def build_probe(force: bool = False) -> str:
-    """tools/philox_roof: the Philox throughput probe bench.py uses as the ALU roof."""
-    src = os.path.join(ROOT, "tools", "philox_roof", "philox_roof.cu")
-    exe = os.path.join(ROOT, "tools", "philox_roof", "philox_roof")
+    """tools/philox_roof: the Philox throughput probe bench.py uses as the ALU
+    roof; tools/gather_roof: the random dependent-load probe (LT walk roof)."""
     hdr = os.path.join(CSRC, "philox.cuh")
-    if force or not os.path.exists(exe) or os.path.getmtime(exe) < max(os.path.getmtime(src), os.path.getmtime(hdr)):
-        subprocess.check_call([_nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "-o", exe, src])
+    exe = ""
+    for name, deps in (("philox_roof", [hdr]), ("gather_roof", [])):
+        src = os.path.join(ROOT, "tools", name, name + ".cu")
+        exe_n = os.path.join(ROOT, "tools", name, name)
+        if force or not os.path.exists(exe_n) or os.path.getmtime(exe_n) < max(os.path.getmtime(p) for p in [src, *deps]):
+            subprocess.check_call([_nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "-o", exe_n, src])
+        exe = exe or exe_n
     return exe
 
 
