@@ -162,6 +162,7 @@ __device__ __forceinline__ unsigned long long gtimer_ns() {
   return t;
 }
 
+template <bool CHUNKED>
 __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   cg::grid_group grid = cg::this_grid();
   __shared__ unsigned long long red[GB / 32];
@@ -180,7 +181,9 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   // decrements, and only those are rescanned (by the block that owns them)
   // before the next argmax.  The keys are exact whenever they are read, so
   // the winner and the tie rule are the full scan's.
-  const bool chunked = nc >= a.chunk_min;
+  // (the chunked argmax is a separate instantiation: the default kernel
+  // carries none of its code)
+  const bool chunked = CHUNKED && nc >= a.chunk_min;
   const uint32_t c4 = (1u << a.chunk_shift) / 4;  // uint4 per chunk (>= 1)
   const uint32_t nchunks = (nc4 + c4 - 1) / c4;
   const uint32_t cpb = (nchunks + gridDim.x - 1) / gridDim.x;  // chunks per block
@@ -188,7 +191,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   for (uint32_t j = 0; j < a.k; ++j) {
     if (a.dbg && blockIdx.x == 0 && threadIdx.x == 0) a.dbg[3 * j] = gtimer_ns();
     unsigned long long km = 0;
-    if (chunked) {
+    if (CHUNKED && chunked) {
       // refresh this block's dirty chunks (a warp per chunk), then reduce
       // its chunk keys
       for (uint32_t c = cb0 + (threadIdx.x >> 5); c < cb1; c += GB / 32) {
@@ -279,7 +282,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         for (uint32_t t = lane; t < L; t += 32) {
           const uint32_t x = a.arena_c[st + t];
           atomicSub(&a.W[x], 1u);
-          if (chunked) a.dirty[x >> a.chunk_shift] = 1;
+          if (CHUNKED && chunked) a.dirty[x >> a.chunk_shift] = 1;
         }
       }
       __syncthreads();
@@ -292,7 +295,7 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
         for (uint32_t t = threadIdx.x; t < L; t += GB) {
           const uint32_t x = a.arena_c[st + t];
           atomicSub(&a.W[x], 1u);
-          if (chunked) a.dirty[x >> a.chunk_shift] = 1;
+          if (CHUNKED && chunked) a.dirty[x >> a.chunk_shift] = 1;
         }
       }
       __syncthreads();
@@ -399,7 +402,9 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   uint8_t* selected = S.covered.as<uint8_t>() + fl_sets;
   uint32_t* zc = reinterpret_cast<uint32_t*>(selected + fl_sel);
   static int per_sm = 0;  // occupancy of the pick kernel (a property of the binary and the device)
-  if (per_sm == 0) EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, greedy_kernel, GB, 0));
+  const char* cm = getenv("EIM_GREEDY_CHUNK_MIN");
+  const void* kern = cm ? (const void*)greedy_kernel<true> : (const void*)greedy_kernel<false>;
+  if (per_sm == 0) EIM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, GB, 0));
   const char* gbe = getenv("EIM_GREEDY_BLOCKS");  // development: grid of the greedy kernel
   uint32_t blocks = gbe ? (uint32_t)atoi(gbe) : (uint32_t)ctx->sm_count;
   // concurrent selections get their share of the SMs (greedy_shares): two
@@ -409,7 +414,6 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   blocks = std::max(1u, std::min(blocks, (uint32_t)std::max(1, per_sm) * ctx->sm_count));
   // chunked argmax from this many candidates on (EIM_GREEDY_CHUNK_MIN; 0:
   // always) with 2^shift candidates per chunk (EIM_GREEDY_CHUNK_SHIFT, >= 2)
-  const char* cm = getenv("EIM_GREEDY_CHUNK_MIN");
   const char* cs = getenv("EIM_GREEDY_CHUNK_SHIFT");
   const uint32_t chunk_shift = std::max<uint32_t>(2, cs ? (uint32_t)strtoul(cs, nullptr, 10) : CHUNK_SHIFT);
   const uint64_t nchunks_max = ((uint64_t)n >> chunk_shift) + 2;
@@ -449,7 +453,7 @@ void greedy_picks(eim_ctx* ctx, int slot, uint32_t n, uint64_t num_sets, uint32_
   if (!S.ev[0])
     for (cudaEvent_t& e : S.ev) EIM_CUDA(cudaEventCreate(&e));
   EIM_CUDA(cudaEventRecord(S.ev[0], st));
-  EIM_CUDA(cudaLaunchCooperativeKernel((void*)greedy_kernel, dim3(blocks), dim3(GB), args, 0, st));
+  EIM_CUDA(cudaLaunchCooperativeKernel(kern, dim3(blocks), dim3(GB), args, 0, st));
   EIM_CUDA(cudaEventRecord(S.ev[1], st));
   ctx->kernel_launches += 2;
   if (a.dbg) {  // file: k, blocks, stamps per pick and block, block 0's stamps, every block's arrivals
