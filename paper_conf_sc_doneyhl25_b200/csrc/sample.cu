@@ -789,6 +789,9 @@ __device__ __forceinline__ uint32_t decide(const RoundView& R, SampleCtl* ctl, u
 
 // The IC sampler of one round: persistent blocks of NSG sub-groups over
 // sample ids [0, count) and the tasks split off heavy samples.
+#ifndef EIM_IDLE_MAX_NS
+#define EIM_IDLE_MAX_NS 2048  // longest back-off of an idle group between polls of the round's control words
+#endif
 #ifndef EIM_IC_THREADS_SM
 #define EIM_IC_THREADS_SM 1280  // resident sampler threads per SM the register budget is cut for
 #endif
@@ -821,7 +824,7 @@ __global__ void __launch_bounds__(G* NSG, ic_min_blocks<G, NSG>()) ic_kernel(GV 
     if (act == ACT_EXIT) break;
     if (act == ACT_IDLE && NSG == 1) {
       if (gtid == 0) __nanosleep(backoff);
-      backoff = min(backoff * 2u, 2048u);
+      backoff = min(backoff * 2u, (uint32_t)EIM_IDLE_MAX_NS);
     } else if (act == ACT_IDLE) {
       // poll the block's jobs (shared memory) for ~backoff ns before the
       // next global poll
