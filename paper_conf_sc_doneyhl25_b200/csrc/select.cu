@@ -173,7 +173,10 @@ __global__ void __launch_bounds__(GB) greedy_kernel(GreedyArgs a) {
   const uint32_t nc4 = ((nc + 3u) & ~3u) / 4;
   const uint4* W4 = reinterpret_cast<const uint4*>(a.W);
   const int lane = threadIdx.x & 31;
-  const uint64_t warp = ((uint64_t)blockIdx.x * GB + threadIdx.x) >> 5;
+  // list entries are dealt to the warps block-interleaved (entry p goes to
+  // block p mod gridDim.x), so a short list spreads over all SMs instead of
+  // filling the first blocks' warps, and long sets do not pile up in one block
+  const uint64_t warp = (uint64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
   const uint64_t nwarps = ((uint64_t)gridDim.x * GB) >> 5;
   // ---- chunked argmax: for many candidates the full scan of W per pick
   // (4 B per candidate from L2/HBM) is replaced by one key per chunk of
