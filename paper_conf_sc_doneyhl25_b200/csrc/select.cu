@@ -36,7 +36,7 @@ namespace {
 
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr int GB = 512;  // threads per block of the greedy kernel
-constexpr uint32_t BIG = 128;      // covered sets with more members are walked by a whole block
+constexpr uint32_t BIG = 64;       // covered sets with more members are walked by a whole block
 constexpr uint32_t BIG_CAP = 256;  // queued per block and pick (more are walked by their warp)
 
 __global__ void flag_kernel(const uint32_t* __restrict__ C, uint32_t n, uint32_t* __restrict__ flags) {
